@@ -1,0 +1,310 @@
+#!/usr/bin/env python
+"""bench.py -- tiled-QR throughput on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
+
+metric : tiled QR GFLOP/s = (2mn^2 - 2n^3/3) / t, whole job, plus % of the FP64 tensor peak.
+step   : one pass of the whole hot path over the config's matrix:
+         tqr_load (col-major -> tiles) + tqr_factor_tiles (GEQRT/TSQRT panels, UNMQR/TSMQR
+         updates, lookahead, broadcasts) + tqr_store_r (R out).  Input resident in HBM.
+e2e    : the same through tqr_factor-equivalent calls on PINNED HOST buffers (H2D of A and
+         D2H of R inside the timed region).
+N > 1  : launched by torchrun; one process per GPU, column tiles partitioned by the guide
+         array {0..N-1} (Eq. 12), panels broadcast with NCCL.  Strong scaling (same matrix).
+--impl reference : the CPU oracle (Algorithm 1, oracle/) timed on this host's cores on a
+         bounded sample of the same workload (first 512 columns of the config's matrix).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (m, n, nb, ib, seed)  -- BASELINE.json configs
+    "C1": (256, 256, 64, 16, 101),
+    "C2": (4096, 4096, 256, 32, 102),
+    "C3": (16384, 16384, 512, 32, 103),
+    "C4": (1048576, 512, 512, 32, 104),
+    "C5": (32768, 32768, 512, 32, 105),
+}
+DEFAULT_CONFIG = "C5"
+L2_BYTES = 126 * 2 ** 20
+
+
+def flops(m, n):
+    return 2.0 * m * n * n - 2.0 * n ** 3 / 3.0
+
+
+def fp64_peak_tflops():
+    """Measured DMMA.8x8x4 peak (profiles/fp64_peak.json, own microbenchmark on this pool)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "fp64_peak.json")) as f:
+            d = json.load(f)
+        return float(d["dmma_tflops"]), d.get("source", "profiles/fp64_peak.json")
+    except Exception:
+        return 37.2, "nominal 148 SM x 64 FMA/clk x 2 x 1.965 GHz"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            try:
+                sm.append(float(r[1]))
+                mx = float(r[2])
+                for i, nm in enumerate(names):
+                    if r[5 + i].lower().startswith("active"):
+                        reasons.add(nm)
+            except Exception:
+                continue
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def oracle_sample(cfg_name, nthreads=0):
+    """Bounded CPU-oracle sample of the config: Algorithm 1 on the first min(n, 512) columns
+    of the config's own matrix (same generator, same rows).  Returns (GFLOP/s, seconds, desc)."""
+    import numpy as np
+    import oracle
+    import synthetic
+    m, n, nb, ib, seed = CONFIGS[cfg_name]
+    ns = min(n, 512)
+    rows = np.arange(m, dtype=np.uint64)
+    A = np.empty((m, ns), order="F")
+    for j in range(ns):
+        A[:, j] = synthetic.gaussian_entries(m, rows, np.full(m, j, dtype=np.uint64), seed)
+    t0 = time.perf_counter()
+    oracle.qr(A, nthreads=nthreads)
+    dt = time.perf_counter() - t0
+    return flops(m, ns) / dt / 1e9, dt, "oracle.qr on A[:, :%d] of %s (%dx%d), %.2f s" % (ns, cfg_name, m, ns, dt)
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, on this host's cores."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    cores = oracle.num_threads()
+    for _ in range(args.warmup):
+        oracle_sample(args.config)
+    vals, times = [], []
+    for _ in range(args.steps):
+        v, dt, desc = oracle_sample(args.config)
+        vals.append(v)
+        times.append(dt)
+    m, n, nb, ib, seed = CONFIGS[args.config]
+    value = statistics.median(vals)
+    line = {
+        "impl": "reference", "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3)", "value": round(value, 3),
+        "unit": "GFLOP/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * statistics.median(times), 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
+                   "sample": "first %d columns" % min(n, 512)},
+        "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": round(value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default=DEFAULT_CONFIG, choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-lookahead", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import paper_conf_icpp_kimp13_b200 as tqr
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local_rank)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+
+    m, n, nb, ib, seed = CONFIGS[args.config]
+    W = max(args.warmup, 3)
+    K = max(args.steps, 1)
+
+    # ---- inputs (seeded synthetic N(0,1), generated on the device; identical on every rank)
+    gen = torch.Generator(device="cuda").manual_seed(seed)
+    A0 = torch.randn((n, m), dtype=torch.float64, device="cuda", generator=gen).t()   # column-major m x n
+    Rout = torch.empty((n, m), dtype=torch.float64, device="cuda").t()
+
+    nccl_id = None
+    if world > 1:
+        obj = [tqr.tqr_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+    plan = tqr.Plan(m, n, nb, ib, ndev=world, rank=rank, world=world, nccl_id=nccl_id,
+                    lookahead=not args.no_lookahead, profile=True)
+
+    def step(Ain, Aout):
+        plan.load(Ain)
+        plan.factor_tiles()
+        plan.store_r(Aout)
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+
+    def max_over_ranks(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    for _ in range(W):
+        step(A0, Rout)
+    torch.cuda.synchronize()
+    plan.kernel_stats(0, reset=True)
+    plan.kernel_stats(1, reset=True)
+    plan.launch_count()
+
+    stream = torch.cuda.current_stream()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for _ in range(K):
+            step(A0, Rout)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    ms = ev0.elapsed_time(ev1) / K
+    ms = max_over_ranks(ms)
+    launches = plan.launch_count() // K
+    ucount, ums, uflops = plan.kernel_stats(0, reset=True)
+    pcount, pms, pflops = plan.kernel_stats(1, reset=True)
+    fl = flops(m, n)
+    value = fl / (ms * 1e-3) / 1e9
+    peak, peak_src = fp64_peak_tflops()
+
+    # ---- e2e: pinned host in, pinned host out, copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        Ah = torch.empty((n, m), dtype=torch.float64, pin_memory=True).t()
+        Ah.copy_(A0)
+        Rh = torch.empty((n, m), dtype=torch.float64, pin_memory=True).t()
+        step(Ah, Rh)
+        torch.cuda.synchronize()
+        barrier()
+        t0 = time.perf_counter()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        ke = max(1, min(K, 2))
+        for _ in range(ke):
+            step(Ah, Rh)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ems = max_over_ranks(e0.elapsed_time(e1) / ke)
+        e2e = {"value": round(fl / (ems * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+               "ms_per_step": round(ems, 3), "h2d_bytes_per_step": 8 * m * n, "d2h_bytes_per_step": 8 * m * n,
+               "api": "tqr_load(host) + tqr_factor_tiles + tqr_store_r(host) == tqr_factor on pinned host A"}
+        del Ah, Rh
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        v, dt, desc = oracle_sample(args.config)
+        cpu = {"value": round(v, 3), "unit": "GFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
+               "sample": desc}
+
+    if rank == 0:
+        upd_ms = ums / max(ucount, 1)
+        upd_fl = uflops / max(ucount, 1)
+        achieved = (upd_fl / (upd_ms * 1e-3) / 1e12) if ucount else None
+        line = {
+            "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak",
+            "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
+            "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "pct_fp64_peak": round(100.0 * value / 1e3 / (peak * world), 2),
+            "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
+                       "input": "torch.randn N(0,1) fp64 on device (seeded)", "guide": list(range(world)),
+                       "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
+                       "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (8 * m * n / 2 ** 30)
+                       if 8 * m * n > L2_BYTES else "input fits L2 (no flush)"},
+            "roofline": {"bound": "tensor", "kernel": "update_kernel (UNMQR+TSMQR, DMMA.8x8x4)",
+                         "achieved": round(achieved, 3) if achieved else None, "peak": peak, "unit": "TFLOP/s",
+                         "frac": round(achieved / peak, 4) if achieved else None, "traffic": None,
+                         "peak_source": peak_src, "launches": ucount, "avg_ms": round(upd_ms, 3),
+                         "share_of_step": round(ums / K / ms, 3) if ucount else None},
+            "panel": {"launches": pcount, "avg_ms": round(pms / max(pcount, 1), 3),
+                      "tflops": round(pflops / max(pms, 1e-9) / 1e9, 3) if pcount else None},
+            "clocks": clk.summary(),
+            "gpu_launches": launches,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    plan.close()
+    if dist is not None:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,165 @@
+/*
+ * tqr.h -- C ABI of the B200-native tiled Householder QR (Kim & Park, ICPP'13).
+ *
+ * Problem statement: A = QR with Q orthogonal (Q^T Q = Q Q^T = I) and R upper
+ * triangular, Eq. (1); A x = b solved as R x = Q^T b, Eqs. (2)-(3) P:L181-188,
+ * P:L242.  The method is the tiled QR of Sec. II.B: Triangulation (GEQRT,
+ * Eqs. 4-5), update for triangulation (UNMQR, Eq. 6, applied as Q^T -- reading Q5),
+ * Elimination (TSQRT, Eqs. 7-8) and update for elimination (TSMQR, Eq. 9), over square
+ * nb x nb tiles.  Column tiles are distributed to devices by the distribution
+ * guide array, Eq. (12) P:L1026 (Algorithm 4).
+ *
+ * Conventions for every entry point:
+ *   - Every call returns tqr_status (TQR_OK = 0).  No C++ exception, abort or exit crosses
+ *     the ABI.  A failed call leaves a message retrievable with tqr_last_error().
+ *   - Matrices are column-major: element (i, j) of X with leading dimension ldx is
+ *     X[i + j*ldx], in the plan's dtype.
+ *   - Pointers may be host memory (pageable or pinned) or device memory of the plan's
+ *     first device; the library detects which with cudaPointerGetAttributes.  The caller
+ *     owns its buffers; the plan never frees or retains them past the call.
+ *   - Calls are synchronous: on return every result is in the caller's buffer.
+ *   - A CUDA or NCCL failure poisons the plan: later calls return TQR_ERR_STATE until
+ *     tqr_destroy.  A plan is not thread-safe; distinct plans are independent.
+ */
+#ifndef TQR_H_
+#define TQR_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tqr_plan_s* tqr_plan;
+
+typedef enum { TQR_F64 = 0, TQR_F32 = 1 } tqr_dtype;
+
+typedef enum {
+    TQR_OK = 0,
+    TQR_ERR_ARG = 1,         /* invalid argument (sizes, guide entries, NULL pointer, ld < m) */
+    TQR_ERR_ALLOC = 2,       /* device or pinned-host allocation failed */
+    TQR_ERR_CUDA = 3,        /* a CUDA runtime call or kernel failed (plan is poisoned) */
+    TQR_ERR_NCCL = 4,        /* NCCL missing or an NCCL call failed (plan is poisoned) */
+    TQR_ERR_STATE = 5,       /* call not valid in the plan's state (e.g. apply before factor) */
+    TQR_ERR_SINGULAR = 6,    /* solve: some R_ii == 0 exactly (LAPACK dtrtrs convention) */
+    TQR_ERR_UNSUPPORTED = 7  /* valid request this build does not implement (dtype/nb/ib combo) */
+} tqr_status;
+
+/* Options for tqr_create_ex.  Zero-initialise, then set what you need. */
+typedef struct {
+    /* 1: all ndev column owners live on the calling thread's current CUDA device
+     * ("logical devices"); panel broadcasts become device-to-device copies.  Exercises the
+     * guide-array partition and broadcast ordering on one GPU.  0: owner d uses CUDA
+     * device d (single-process) or this process's device (multi-process). */
+    int32_t logical_devices;
+    /* Multi-process mode (one process per GPU): world > 1, this process is `rank`; ndev must
+     * equal world.  nccl_id points to the 128-byte ncclUniqueId produced by
+     * tqr_nccl_unique_id() on rank 0 and shared out of band (e.g. torch.distributed). */
+    int32_t rank;
+    int32_t world;
+    const void* nccl_id;
+    /* 0 = disable the one-panel lookahead (plain step order), otherwise enabled (default). */
+    int32_t no_lookahead;
+    /* 1: record CUDA events around every update-kernel launch so tqr_kernel_stats() can
+     * report the dominant kernel's device time (bench.py roofline). */
+    int32_t profile;
+} tqr_options;
+
+/*
+ * Create a plan for the QR factorisation of an m x n matrix.
+ *   m, n      : matrix size, m >= n >= 1; this build needs m % nb == 0 and n % nb == 0.
+ *   nb        : tile size (square tiles); supported 64, 128, 256, 512.
+ *   ib        : inner blocking of the compact-WY T factors; 1 <= ib <= nb, nb % ib == 0;
+ *               supported 16, 32.
+ *   dtype     : TQR_F64 (TQR_F32 returns TQR_ERR_UNSUPPORTED in this build).
+ *   ndev      : number of column-tile owners (devices).
+ *   guide     : distribution guide array (Alg. 4), entries in [0, ndev); column tile j is
+ *               owned by guide[j % guide_len] (Eq. 12).  NULL -> {0, 1, ..., ndev-1}.
+ *   out       : receives the plan (owned by the caller, release with tqr_destroy).
+ * The plan owns all device memory (tile storage, T factors, panel receive buffers),
+ * streams, events and (multi-process) the NCCL communicator.
+ * Errors: TQR_ERR_ARG on invalid sizes/guide, TQR_ERR_UNSUPPORTED on unsupported combos,
+ * TQR_ERR_ALLOC / TQR_ERR_CUDA / TQR_ERR_NCCL on resource failures (nothing is leaked).
+ */
+tqr_status tqr_create(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype,
+                      int32_t ndev, const int32_t* guide, int32_t guide_len, tqr_plan* out);
+
+/* As tqr_create with explicit options (opt may be NULL = all defaults). */
+tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype,
+                         int32_t ndev, const int32_t* guide, int32_t guide_len,
+                         const tqr_options* opt, tqr_plan* out);
+
+/*
+ * Factor A (m x n, lda >= m) in place: A = QR (Eq. 1).  On return A(0:n, 0:n) holds R in
+ * its upper triangle and every entry below the diagonal of A is zero (the reflectors stay
+ * inside the plan in tile layout for tqr_apply_qt / tqr_solve_ls).  In multi-process mode
+ * A is the full matrix on every rank and each rank writes back the columns it owns.
+ * The call runs a1 (layout convert), a2-a7 (tiled factorisation) and a8 (R out).
+ */
+tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda);
+
+/* The three phases of tqr_factor, for timing: tiles <- A; factor the resident tiles;
+ * A <- R.  tqr_factor == tqr_load + tqr_factor_tiles + tqr_store_r. */
+tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda);
+tqr_status tqr_factor_tiles(tqr_plan h);
+tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda);
+
+/*
+ * B (m x nrhs, ldb >= m) <- Q^T B (trans 'T') or Q B (trans 'N'), with Q from the last
+ * tqr_factor (Alg. 1 lines 13-14 read for the tiled factorisation).  Rows 0..n-1 of Q^T B
+ * (and Q [C; 0]) are unique; rows n..m-1 of Q^T B depend on the tile algorithm.
+ * TQR_ERR_STATE before a successful factor.  Multi-process plans: TQR_ERR_UNSUPPORTED.
+ */
+tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs);
+
+/*
+ * Least squares min ||A X - B||_F via Eqs. (2)-(3): B <- Q^T B, then R X = B(0:n, :) by
+ * back substitution; X is returned in B(0:n, :) (rows n..m-1 unspecified).
+ * TQR_ERR_SINGULAR if some R_ii == 0 exactly (B unspecified).
+ */
+tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs);
+
+/* Release everything the plan owns.  NULL-safe; always TQR_OK for a valid or NULL plan. */
+tqr_status tqr_destroy(tqr_plan h);
+
+/* Static description of a status code. */
+const char* tqr_status_string(tqr_status s);
+
+/* Message of the last failed call on h (or of the last failed tqr_create when h is NULL). */
+const char* tqr_last_error(tqr_plan h);
+
+/* Write a fresh 128-byte ncclUniqueId into id[0..127] (rank 0 of a multi-process plan).
+ * TQR_ERR_NCCL if libnccl.so.2 cannot be loaded. */
+tqr_status tqr_nccl_unique_id(void* id128);
+
+/* Owner of column tile j under the plan's guide array (Eq. 12), or -1 if j is out of range. */
+int32_t tqr_owner(tqr_plan h, int64_t j);
+
+/*
+ * Host-side schedule of the tiled DAG (Fig. 3) for rank `rank`: writes up to
+ * cap records of 5 int32 {op, k, i, j, root} into ops and the total count into *count.
+ * op: 0 = PANEL (GEQRT(k,k) + TSQRT(i,k) chain, on owner(k)), 1 = BCAST (panel k from
+ * root = owner(k)), 2 = UPDATE (UNMQR(k,j) + TSMQR(i,j,k) chain for column j).  Pure host
+ * logic (no GPU needed); used by the multi-process CPU tests.
+ */
+tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const int32_t* guide,
+                        int32_t guide_len, int32_t rank, int32_t* ops, int64_t cap, int64_t* count);
+
+/* Distribution guide array from integer per-device tile-update rates (Alg. 4 GET_RATIO +
+ * GENERATE_ARRAY; ties -> lowest ID).  Writes sum(ratio) entries to guide
+ * (capacity cap) and the length to *len. */
+tqr_status tqr_generate_guide(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len);
+
+/* Device-time statistics of the plan's kernels since the last reset (opt.profile = 1):
+ * which = 0 update (UNMQR+TSMQR) kernel, 1 panel (GEQRT+TSQRT) kernel, 2 layout kernels,
+ * 3 broadcast.  *count launches, *ms summed CUDA-event milliseconds, *flops algorithmic
+ * flops of those launches.  reset != 0 clears after reading. */
+tqr_status tqr_kernel_stats(tqr_plan h, int32_t which, int64_t* count, double* ms, double* flops, int32_t reset);
+
+/* Number of kernel launches the plan issued since the last call (then resets). */
+int64_t tqr_launch_count(tqr_plan h);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TQR_H_ */

@@ -1,0 +1,352 @@
+// qr_kernels.cu -- the sm_100a hot path of the tiled Householder QR.
+//
+//   panel_kernel  : GEQRT(k,k) followed by the flat-TS chain TSQRT(i,k), i = k+1..p-1
+//                   (Eqs. 4-5, 7-8; Fig. 3 DAG P:L332-345; reading Q7: flat,
+//                   top-down).  One CTA per ib-wide column block of panel k; CTA b applies
+//                   the reflector blocks b' < b of tile i as soon as CTA b' publishes them
+//                   (inter-CTA release/acquire flags), then factors its own block.  The chain
+//                   over i therefore runs as a wavefront across the NB/IB CTAs.
+//   update_kernel : UNMQR(k,j) + TSMQR(i,j,k), i = k+1..p-1, for every trailing column j
+//                   (Eqs. 6 and 9).  One CTA per W-wide column slice; the slice of A_ij lives
+//                   in registers for all ib blocks of Q_ik, A_kj stays L2-resident as the
+//                   "top" row block of every TS pair.  Also used (TRANS / reverse order) for
+//                   Q^T B and Q B in tqr_apply_qt.
+//   layout kernels: column-major <-> tile-major (128-bit when aligned), R out with zeroed
+//                   lower part, and the back substitution of tqr_solve_ls (Eq. 3).
+#include <cstdio>
+#include "tile_ops.cuh"
+#include "../tqr_internal.h"
+
+namespace tqr {
+
+// ============================================================================ panel kernel
+template <int NB, int IB>
+__global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    auto& sm = *reinterpret_cast<Smem<NB, IB, IB>*>(smem_raw);
+    constexpr int NBLK = NB / IB;
+    const int b = blockIdx.x;
+    const int64_t tile = (int64_t)NB * NB;
+    double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
+    double* Akk = col + (int64_t)a.k * tile;
+    Slice<NB, IB, IB> X;
+
+    for (int i = a.k; i < a.p; ++i) {
+        double* Ai = col + (int64_t)i * tile;
+        double* Ti = a.T + (int64_t)i * IB * NB;
+        const bool ge = (i == a.k);
+        X.load_cg(Ai + (int64_t)b * IB * NB, NB);
+        for (int bp = 0; bp < b; ++bp) {
+            flag_wait_geq(a.flags + (int64_t)i * NBLK + bp, a.epoch);
+            if (ge)
+                apply_block<NB, IB, IB, true, true>(X, sm, a.Vexp + (int64_t)bp * IB * NB, NB,
+                                                    Ti + (int64_t)bp * IB * IB, nullptr, 0, bp * IB);
+            else
+                apply_block<NB, IB, IB, true, true>(X, sm, Ai + (int64_t)bp * IB * NB, NB,
+                                                    Ti + (int64_t)bp * IB * IB,
+                                                    Akk + (int64_t)b * IB * NB + bp * IB, NB, 0);
+        }
+        if (ge) {
+            factor_block<NB, IB, true>(X, sm, b * IB);
+        } else {
+            // diagonal R block of this column block: R(b*IB + c, b*IB + j), upper triangle
+            for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+                const int c = idx / IB, j = idx % IB;
+                sm.Rsm[c * IB + j] = (j >= c) ? ld_cg(Akk + (int64_t)(b * IB + j) * NB + b * IB + c) : 0.0;
+            }
+            __syncthreads();
+            factor_block<NB, IB, false>(X, sm, b * IB);
+        }
+        // publish: reflectors, T block, R block (TSQRT), explicit V (GEQRT)
+        X.store(Ai + (int64_t)b * IB * NB, NB);
+        for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+            const int c = idx / IB, r = idx % IB;   // T(r, c) -> column-major block b
+            Ti[(int64_t)b * IB * IB + c * IB + r] = sm.Tsm[r * IB + c];
+        }
+        if (ge) {
+            const int g = lane_id() >> 2, t = lane_id() & 3, r0 = warp_id() * (NB / 8) + 2 * t;
+#pragma unroll
+            for (int mf = 0; mf < IB / 8; ++mf) {
+                const int dc = b * IB + mf * 8 + g;
+#pragma unroll
+                for (int nf = 0; nf < NB / 64; ++nf) {
+                    const int r = r0 + nf * 8;
+                    double v0 = (r > dc) ? X.acc[mf][nf][0] : (r == dc ? 1.0 : 0.0);
+                    double v1 = (r + 1 > dc) ? X.acc[mf][nf][1] : (r + 1 == dc ? 1.0 : 0.0);
+                    st2(a.Vexp + (int64_t)dc * NB + r, v0, v1);
+                }
+            }
+        } else {
+            for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+                const int j = idx / IB, c = idx % IB;
+                if (c <= j) Akk[(int64_t)(b * IB + j) * NB + b * IB + c] = sm.Rsm[c * IB + j];
+            }
+        }
+        __threadfence();
+        __syncthreads();
+        if (threadIdx.x == 0) flag_release(a.flags + (int64_t)i * NBLK + b, a.epoch);
+    }
+}
+
+// ============================================================================ update kernel
+// Forward (TRANS = true, Q^T): for each slice: [UNMQR on row tile k]; for i = k+1..p-1 TSMQR.
+// Backward (TRANS = false, Q):  for i = p-1..k+1 TSMQR (blocks descending); then UNMQR.
+template <int NB, int W, int IB, bool TRANS>
+__global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    auto& sm = *reinterpret_cast<Smem<NB, W, IB>*>(smem_raw);
+    constexpr int SPG = NB / W;     // slices per column group
+    constexpr int NBLK = NB / IB;
+    const int grp = blockIdx.x / SPG;
+    const int c0 = (blockIdx.x % SPG) * W;
+    double* Xg = a.X + (int64_t)(a.group0 + grp) * a.col_stride + (int64_t)c0 * a.ld;
+    double* Xk = Xg + (int64_t)a.k * a.tile_stride;
+    const int64_t vtile = (int64_t)NB * NB;
+    Slice<NB, W, IB> X;
+
+    auto unmqr = [&]() {
+        X.load(Xk, a.ld);
+        const double* Tk = a.T + (int64_t)a.k * IB * NB;
+        if (TRANS) {
+            for (int s = 0; s < NBLK; ++s)
+                apply_block<NB, W, IB, TRANS, false>(X, sm, a.Vexp + (int64_t)s * IB * NB, NB,
+                                                     Tk + (int64_t)s * IB * IB, nullptr, 0, s * IB);
+        } else {
+            for (int s = NBLK - 1; s >= 0; --s)
+                apply_block<NB, W, IB, TRANS, false>(X, sm, a.Vexp + (int64_t)s * IB * NB, NB,
+                                                     Tk + (int64_t)s * IB * IB, nullptr, 0, s * IB);
+        }
+        X.store(Xk, a.ld);
+        __syncthreads();
+    };
+    auto tsmqr = [&](int i) {
+        double* Xi = Xg + (int64_t)i * a.tile_stride;
+        const double* Vi = a.V + (int64_t)i * vtile;
+        const double* Ti = a.T + (int64_t)i * IB * NB;
+        X.load(Xi, a.ld);
+        if (TRANS) {
+            for (int s = 0; s < NBLK; ++s)
+                apply_block<NB, W, IB, TRANS, false>(X, sm, Vi + (int64_t)s * IB * NB, NB,
+                                                     Ti + (int64_t)s * IB * IB, Xk + s * IB, a.ld, 0);
+        } else {
+            for (int s = NBLK - 1; s >= 0; --s)
+                apply_block<NB, W, IB, TRANS, false>(X, sm, Vi + (int64_t)s * IB * NB, NB,
+                                                     Ti + (int64_t)s * IB * IB, Xk + s * IB, a.ld, 0);
+        }
+        X.store(Xi, a.ld);
+    };
+
+    if (TRANS) {
+        if (a.do_unmqr) unmqr();
+        for (int i = a.k + 1; i < a.p; ++i) tsmqr(i);
+    } else {
+        for (int i = a.p - 1; i > a.k; --i) tsmqr(i);
+        __syncthreads();
+        if (a.do_unmqr) unmqr();
+    }
+}
+
+// ============================================================================ layout kernels
+// a1: column-major source -> tile-major column storage.  Source column group of local column
+// lc starts at src + cols[lc]*src_group_stride (ld = lda); destination tile i of local column
+// lc at dst + lc*dst_col_stride + i*nb*nb, element (r, c) at + c*nb + r.  blockIdx.x = chunk*nb
+// + c, blockIdx.y = lc.  128-bit (double2) when lda and the pointer are 16-byte aligned: a warp
+// moves 512 contiguous bytes per instruction on both sides.
+__global__ void to_tiles_kernel(const double* __restrict__ src, int64_t lda, int64_t src_group_stride,
+                                double* __restrict__ dst, const int32_t* __restrict__ cols,
+                                int64_t dst_col_stride, int nb, int p, int vec2) {
+    const int lc = blockIdx.y;
+    const int c = blockIdx.x % nb;
+    const int chunk = blockIdx.x / nb, nchunk = gridDim.x / nb;
+    const double* s = src + (int64_t)(cols ? cols[lc] : lc) * src_group_stride + (int64_t)c * lda;
+    double* d = dst + (int64_t)lc * dst_col_stride + (int64_t)c * nb;
+    const int64_t tile = (int64_t)nb * nb;
+    const int64_t m = (int64_t)p * nb;
+    if (vec2) {
+        for (int64_t r = 2 * ((int64_t)chunk * blockDim.x + threadIdx.x); r < m; r += 2 * (int64_t)nchunk * blockDim.x) {
+            const double2 v = __ldcs(reinterpret_cast<const double2*>(s + r));
+            *reinterpret_cast<double2*>(d + (r / nb) * tile + (r % nb)) = v;
+        }
+    } else {
+        for (int64_t r = (int64_t)chunk * blockDim.x + threadIdx.x; r < m; r += (int64_t)nchunk * blockDim.x)
+            d[(r / nb) * tile + (r % nb)] = s[r];
+    }
+}
+
+// a8: tile-major -> column-major rows [0, m_rows): R on and above the diagonal, 0 below.
+__global__ void from_tiles_kernel(double* __restrict__ dst, int64_t lda, int64_t dst_group_stride,
+                                  const double* __restrict__ src, const int32_t* __restrict__ cols,
+                                  int64_t src_col_stride, int nb, int64_t m_rows, int local_dst, int vec2) {
+    const int lc = blockIdx.y;
+    const int c = blockIdx.x % nb;
+    const int chunk = blockIdx.x / nb, nchunk = gridDim.x / nb;
+    const int64_t gcol = (int64_t)cols[lc] * nb + c;
+    double* d = dst + (int64_t)(local_dst ? lc : cols[lc]) * dst_group_stride + (int64_t)c * lda;
+    const double* s = src + (int64_t)lc * src_col_stride + (int64_t)c * nb;
+    const int64_t tile = (int64_t)nb * nb;
+    if (vec2) {
+        for (int64_t r = 2 * ((int64_t)chunk * blockDim.x + threadIdx.x); r < m_rows; r += 2 * (int64_t)nchunk * blockDim.x) {
+            double2 v = make_double2(0.0, 0.0);
+            if (r <= gcol) {
+                v = *reinterpret_cast<const double2*>(s + (r / nb) * tile + (r % nb));
+                if (r + 1 > gcol) v.y = 0.0;
+            }
+            __stcs(reinterpret_cast<double2*>(d + r), v);
+        }
+    } else {
+        for (int64_t r = (int64_t)chunk * blockDim.x + threadIdx.x; r < m_rows; r += (int64_t)nchunk * blockDim.x)
+            d[r] = (r <= gcol) ? s[(r / nb) * tile + (r % nb)] : 0.0;
+    }
+}
+
+// Back substitution R X = C for the n x n upper-triangular R held in tile layout (panel
+// column owner storage gathered into `Rcm`, column-major n x n, ld = ldr).  One CTA per
+// right-hand side; columns of R are streamed (Eq. 3).
+__global__ void trsv_upper_kernel(const double* __restrict__ R, int64_t ldr, double* __restrict__ C,
+                                  int64_t ldc, int64_t n) {
+    double* x = C + (int64_t)blockIdx.x * ldc;
+    __shared__ double xi_s;
+    for (int64_t i = n - 1; i >= 0; --i) {
+        if (threadIdx.x == 0) xi_s = x[i] / R[i + i * ldr];
+        __syncthreads();
+        const double xi = xi_s;
+        const double* rc = R + i * ldr;
+        for (int64_t r = threadIdx.x; r < i; r += blockDim.x) x[r] -= rc[r] * xi;
+        if (threadIdx.x == 0) x[i] = xi;
+        __syncthreads();
+    }
+}
+
+__global__ void zero_diag_check_kernel(const double* __restrict__ R, int64_t ldr, int64_t n, int64_t* first_zero) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (R[i + i * ldr] == 0.0) atomicMin(reinterpret_cast<unsigned long long*>(first_zero), (unsigned long long)i);
+}
+
+// ============================================================================ launchers
+template <int NB, int IB>
+static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s) {
+    const size_t smem = sizeof(Smem<NB, IB, IB>);
+    auto kern = panel_kernel<NB, IB>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<NB / IB, kThreads, smem, s>>>(a);
+    return cudaGetLastError();
+}
+
+template <int NB, int W, int IB>
+static cudaError_t launch_update_t(const UpdateArgs& a, int nslices, bool trans, cudaStream_t s) {
+    const size_t smem = sizeof(Smem<NB, W, IB>);
+    const int grid = nslices;
+    if (grid <= 0) return cudaSuccess;
+    if (trans) {
+        auto kern = update_kernel<NB, W, IB, true>;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        kern<<<grid, kThreads, smem, s>>>(a);
+    } else {
+        auto kern = update_kernel<NB, W, IB, false>;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        kern<<<grid, kThreads, smem, s>>>(a);
+    }
+    return cudaGetLastError();
+}
+
+#define TQR_NBIB_DISPATCH(NB_, IB_, CALL)                              \
+    if (nb == NB_ && ib == IB_) { return CALL; }
+
+cudaError_t launch_panel(int nb, int ib, const PanelArgs& a, cudaStream_t s) {
+    TQR_NBIB_DISPATCH(64, 16, (launch_panel_t<64, 16>(a, s)))
+    TQR_NBIB_DISPATCH(64, 32, (launch_panel_t<64, 32>(a, s)))
+    TQR_NBIB_DISPATCH(128, 16, (launch_panel_t<128, 16>(a, s)))
+    TQR_NBIB_DISPATCH(128, 32, (launch_panel_t<128, 32>(a, s)))
+    TQR_NBIB_DISPATCH(256, 16, (launch_panel_t<256, 16>(a, s)))
+    TQR_NBIB_DISPATCH(256, 32, (launch_panel_t<256, 32>(a, s)))
+    TQR_NBIB_DISPATCH(512, 16, (launch_panel_t<512, 16>(a, s)))
+    TQR_NBIB_DISPATCH(512, 32, (launch_panel_t<512, 32>(a, s)))
+    return cudaErrorInvalidValue;
+}
+
+// w: slice width (8, 16, 32).  Narrow slices raise CTA count for the lookahead column.
+cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslices, bool trans, cudaStream_t s) {
+#define TQR_UPD(NB_, IB_)                                                                 \
+    if (nb == NB_ && ib == IB_) {                                                         \
+        if (w == 8) return launch_update_t<NB_, 8, IB_>(a, nslices, trans, s);            \
+        if (w == 16) return launch_update_t<NB_, 16, IB_>(a, nslices, trans, s);          \
+        if (w == 32) return launch_update_t<NB_, 32, IB_>(a, nslices, trans, s);          \
+        return cudaErrorInvalidValue;                                                     \
+    }
+    TQR_UPD(64, 16)
+    TQR_UPD(64, 32)
+    TQR_UPD(128, 16)
+    TQR_UPD(128, 32)
+    TQR_UPD(256, 16)
+    TQR_UPD(256, 32)
+    TQR_UPD(512, 16)
+    TQR_UPD(512, 32)
+#undef TQR_UPD
+    return cudaErrorInvalidValue;
+}
+
+static int layout_chunks(int64_t m, int vec2, int threads) {
+    int64_t chunks = (m / (vec2 ? 2 : 1) + threads - 1) / threads;
+    return (int)(chunks > 16 ? 16 : (chunks < 1 ? 1 : chunks));
+}
+
+cudaError_t launch_to_tiles(const double* src, int64_t lda, int64_t src_group_stride, double* dst,
+                            const int32_t* cols_dev, int ncols, int64_t dst_col_stride, int nb, int p,
+                            cudaStream_t s) {
+    if (ncols <= 0) return cudaSuccess;
+    const int vec2 = ((lda % 2) == 0 && (src_group_stride % 2) == 0 && (((uintptr_t)src) % 16) == 0) ? 1 : 0;
+    const int threads = 256;
+    dim3 grid(nb * layout_chunks((int64_t)p * nb, vec2, threads), ncols);
+    to_tiles_kernel<<<grid, threads, 0, s>>>(src, lda, src_group_stride, dst, cols_dev, dst_col_stride, nb, p, vec2);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_from_tiles(double* dst, int64_t lda, int64_t dst_group_stride, const double* src,
+                              const int32_t* cols_dev, int ncols, int64_t src_col_stride, int nb, int p,
+                              int64_t m_rows, int local_dst, cudaStream_t s) {
+    (void)p;
+    if (ncols <= 0 || m_rows <= 0) return cudaSuccess;
+    const int vec2 = ((lda % 2) == 0 && (dst_group_stride % 2) == 0 && (m_rows % 2) == 0 &&
+                      (((uintptr_t)dst) % 16) == 0) ? 1 : 0;
+    const int threads = 256;
+    dim3 grid(nb * layout_chunks(m_rows, vec2, threads), ncols);
+    from_tiles_kernel<<<grid, threads, 0, s>>>(dst, lda, dst_group_stride, src, cols_dev, src_col_stride, nb,
+                                               m_rows, local_dst, vec2);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_trsv_upper(const double* R, int64_t ldr, double* C, int64_t ldc, int64_t n, int64_t nrhs,
+                              cudaStream_t s) {
+    if (nrhs <= 0) return cudaSuccess;
+    trsv_upper_kernel<<<(unsigned)nrhs, 256, 0, s>>>(R, ldr, C, ldc, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_zero_diag_check(const double* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s) {
+    zero_diag_check_kernel<<<64, 256, 0, s>>>(R, ldr, n, first_zero);
+    return cudaGetLastError();
+}
+
+size_t panel_smem_bytes(int nb, int ib) {
+#define TQR_PS(NB_, IB_) if (nb == NB_ && ib == IB_) return sizeof(Smem<NB_, IB_, IB_>);
+    TQR_PS(64, 16) TQR_PS(64, 32) TQR_PS(128, 16) TQR_PS(128, 32)
+    TQR_PS(256, 16) TQR_PS(256, 32) TQR_PS(512, 16) TQR_PS(512, 32)
+#undef TQR_PS
+    return 0;
+}
+
+size_t update_smem_bytes(int nb, int ib, int w) {
+#define TQR_US(NB_, IB_) if (nb == NB_ && ib == IB_) { \
+        if (w == 8) return sizeof(Smem<NB_, 8, IB_>); \
+        if (w == 16) return sizeof(Smem<NB_, 16, IB_>); \
+        if (w == 32) return sizeof(Smem<NB_, 32, IB_>); }
+    TQR_US(64, 16) TQR_US(64, 32) TQR_US(128, 16) TQR_US(128, 32)
+    TQR_US(256, 16) TQR_US(256, 32) TQR_US(512, 16) TQR_US(512, 32)
+#undef TQR_US
+    return 0;
+}
+
+}  // namespace tqr

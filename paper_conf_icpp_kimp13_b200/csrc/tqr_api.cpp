@@ -1,0 +1,831 @@
+// tqr_api.cpp -- C ABI (include/tqr.h), plan/partition, tile-DAG scheduler on CUDA streams.
+//
+// Partition (Sec. IV.C): column tiles are owned per the distribution guide array,
+// owner(j) = guide[j % len] (Eq. 12; reading Q13: every column, owner-computes).
+// Tiles of an owned column are contiguous in the owner's HBM (tile (i, j) is nb x nb
+// column-major), so panel k's reflectors (tiles k..p-1), T factors and explicit V are three
+// contiguous ranges that are broadcast without packing.
+//
+// Schedule (Fig. 3 DAG; Sec. IV.D progress P:L1028-1039, re-designed): per step k
+//   owner(k), panel stream : PANEL(k) = GEQRT(k,k) + TSQRT(k+1..p-1, k)       -> ev_panel[k]
+//   every other owner d    : comm stream receives panel k (peer copy or ncclBroadcast)
+//   owner(k+1), panel str. : lookahead UPDATE(k, column k+1) (waits rest(k-1))   -> ev_look[k]
+//   every owner d, upd str.: UPDATE(k, its columns > k except the lookahead one) -> ev_upd[k]
+// so PANEL(k+1) overlaps the bulk trailing update of step k.  The panel stream has the
+// highest stream priority so freed SMs go to the critical path first.
+#include "../../include/tqr.h"
+
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "nccl_dl.h"
+#include "tqr_internal.h"
+
+using tqr::PanelArgs;
+using tqr::UpdateArgs;
+
+namespace {
+
+thread_local std::string g_create_error;
+
+struct Owner {
+    int id = 0;
+    int dev = 0;
+    std::vector<int32_t> cols;      // global column tiles owned (ascending)
+    std::vector<int32_t> lidx;      // global j -> local index or -1
+    int32_t* cols_dev = nullptr;
+    double* tiles = nullptr;        // ncols * p * nb*nb
+    double* T = nullptr;            // ncols * p * ib*nb
+    double* Vexp = nullptr;         // ncols * nb*nb
+    double* rb_tiles[2] = {nullptr, nullptr};
+    double* rb_T[2] = {nullptr, nullptr};
+    double* rb_V[2] = {nullptr, nullptr};
+    unsigned* flags = nullptr;      // p * (nb/ib)
+    double* io = nullptr;           // m x (nb*ncols) column-major mirror for host / remote I/O
+    cudaStream_t s_panel = nullptr, s_upd = nullptr, s_comm = nullptr;
+    std::vector<cudaEvent_t> ev_panel, ev_recv, ev_upd, ev_look;
+    std::vector<cudaEvent_t> tm0, tm1, tp0, tp1;   // profiling pairs (update rest / panel)
+    std::vector<char> tm_used, tp_used;
+};
+
+struct KStat {
+    int64_t count = 0;
+    double ms = 0.0, flops = 0.0;
+};
+
+}  // namespace
+
+struct tqr_plan_s {
+    int64_t m = 0, n = 0;
+    int nb = 0, ib = 0, p = 0, q = 0;
+    tqr_dtype dtype = TQR_F64;
+    int ndev = 1;
+    std::vector<int32_t> guide;
+    std::vector<int32_t> owner_of;  // size q
+    bool logical = false;
+    int rank = 0, world = 1;
+    bool lookahead = true, profile = false;
+    std::vector<Owner> owners;      // in-process: ndev entries; multi-process: 1 (this rank)
+    const tqr::NcclApi* nccl = nullptr;
+    ncclComm_t comm = nullptr;
+    bool factored = false, poisoned = false;
+    unsigned epoch = 1;
+    std::string err;
+    KStat stats[4];
+    int64_t launches = 0;
+    // apply / solve workspace (single-device plans)
+    double* bw = nullptr;
+    size_t bw_elems = 0;
+    double* rcm = nullptr;
+    int64_t* dflag = nullptr;
+
+    bool multiproc() const { return world > 1; }
+    Owner* local(int d) {
+        if (multiproc()) return (d == rank) ? &owners[0] : nullptr;
+        return &owners[d];
+    }
+};
+
+namespace {
+
+tqr_status fail(tqr_plan h, tqr_status st, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    if (h) {
+        h->err = buf;
+        if (st == TQR_ERR_CUDA || st == TQR_ERR_NCCL) h->poisoned = true;
+    } else {
+        g_create_error = buf;
+    }
+    return st;
+}
+
+#define CUDA_TRY(h, call)                                                                          \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess)                                                                     \
+            return fail((h), TQR_ERR_CUDA, "%s:%d %s -> %s", __FILE__, __LINE__, #call,            \
+                        cudaGetErrorString(e_));                                                   \
+    } while (0)
+
+#define NCCL_TRY(h, call)                                                                          \
+    do {                                                                                           \
+        ncclResult_t r_ = (call);                                                                  \
+        if (r_ != ncclSuccess)                                                                     \
+            return fail((h), TQR_ERR_NCCL, "%s:%d %s -> %s", __FILE__, __LINE__, #call,            \
+                        (h)->nccl->GetErrorString(r_));                                            \
+    } while (0)
+
+bool supported_nb_ib(int nb, int ib) {
+    return (nb == 64 || nb == 128 || nb == 256 || nb == 512) && (ib == 16 || ib == 32) && ib <= nb;
+}
+
+// Slice width of the bulk update kernel and of the (latency-critical) lookahead column.
+int w_bulk(const tqr_plan_s*) { return 32; }
+int w_look(const tqr_plan_s* h) { return h->nb >= 256 ? 8 : 16; }
+
+double flops_update(const tqr_plan_s* h, int k, int ncols) {
+    const double nb3 = (double)h->nb * h->nb * h->nb;
+    return (double)ncols * (2.0 * nb3 + 4.0 * nb3 * (double)(h->p - k - 1));
+}
+double flops_panel(const tqr_plan_s* h, int k) {
+    const double nb3 = (double)h->nb * h->nb * h->nb;
+    return 4.0 / 3.0 * nb3 + 2.0 * nb3 * (double)(h->p - k - 1);
+}
+
+void free_owner(Owner& o) {
+    cudaSetDevice(o.dev);
+    auto F = [](void* p) { if (p) cudaFree(p); };
+    F(o.cols_dev); F(o.tiles); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
+    for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
+    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_upd, &o.ev_look, &o.tm0, &o.tm1, &o.tp0, &o.tp1})
+        for (auto e : *v) if (e) cudaEventDestroy(e);
+    if (o.s_panel) cudaStreamDestroy(o.s_panel);
+    if (o.s_upd) cudaStreamDestroy(o.s_upd);
+    if (o.s_comm) cudaStreamDestroy(o.s_comm);
+}
+
+// Host-side DAG (Fig. 3) per rank, the same order the executor issues.
+void build_schedule(int64_t q, const std::vector<int32_t>& owner_of, int rank, std::vector<int32_t>& out) {
+    for (int k = 0; k < q; ++k) {
+        const int o = owner_of[k];
+        if (o == rank) { out.insert(out.end(), {0, k, k, k, o}); }
+        out.insert(out.end(), {1, k, k, k, o});
+        for (int j = k + 1; j < q; ++j)
+            if (owner_of[j] == rank) out.insert(out.end(), {2, k, k, j, o});
+    }
+}
+
+std::vector<int32_t> generate_guide(const std::vector<int32_t>& rates) {
+    // GET_RATIO: divide by the gcd; GENERATE_ARRAY: argmax + decrement,
+    // lowest ID on ties (readings Q11/Q12).
+    int g = 0;
+    for (int r : rates) g = std::gcd(g, r);
+    std::vector<int32_t> ratio(rates.size());
+    int sum = 0;
+    for (size_t i = 0; i < rates.size(); ++i) { ratio[i] = rates[i] / g; sum += ratio[i]; }
+    std::vector<int32_t> ga(sum);
+    for (int i = 0; i < sum; ++i) {
+        int best = 0;
+        for (int d = 1; d < (int)ratio.size(); ++d) if (ratio[d] > ratio[best]) best = d;
+        ga[i] = best;
+        ratio[best] -= 1;
+    }
+    return ga;
+}
+
+enum class Mem { Host, Device };
+struct PtrInfo { Mem kind; int dev; };
+
+PtrInfo classify(const void* p) {
+    cudaPointerAttributes at;
+    cudaError_t e = cudaPointerGetAttributes(&at, p);
+    if (e != cudaSuccess) { cudaGetLastError(); return {Mem::Host, -1}; }
+    if (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged) return {Mem::Device, at.device};
+    return {Mem::Host, -1};
+}
+
+tqr_status ensure_io(tqr_plan h, Owner& o) {
+    if (o.io || o.cols.empty()) return TQR_OK;
+    CUDA_TRY(h, cudaSetDevice(o.dev));
+    CUDA_TRY(h, cudaMalloc(&o.io, sizeof(double) * (size_t)h->m * h->nb * o.cols.size()));
+    return TQR_OK;
+}
+
+tqr_status sync_all(tqr_plan h) {
+    for (auto& o : h->owners) {
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        CUDA_TRY(h, cudaStreamSynchronize(o.s_panel));
+        CUDA_TRY(h, cudaStreamSynchronize(o.s_upd));
+        CUDA_TRY(h, cudaStreamSynchronize(o.s_comm));
+    }
+    return TQR_OK;
+}
+
+}  // namespace
+
+// ================================================================================= ABI
+extern "C" {
+
+const char* tqr_status_string(tqr_status s) {
+    switch (s) {
+        case TQR_OK: return "TQR_OK";
+        case TQR_ERR_ARG: return "TQR_ERR_ARG: invalid argument";
+        case TQR_ERR_ALLOC: return "TQR_ERR_ALLOC: allocation failed";
+        case TQR_ERR_CUDA: return "TQR_ERR_CUDA: CUDA error";
+        case TQR_ERR_NCCL: return "TQR_ERR_NCCL: NCCL error";
+        case TQR_ERR_STATE: return "TQR_ERR_STATE: invalid state";
+        case TQR_ERR_SINGULAR: return "TQR_ERR_SINGULAR: R has a zero diagonal entry";
+        case TQR_ERR_UNSUPPORTED: return "TQR_ERR_UNSUPPORTED: not supported by this build";
+    }
+    return "unknown tqr_status";
+}
+
+const char* tqr_last_error(tqr_plan h) { return h ? h->err.c_str() : g_create_error.c_str(); }
+
+tqr_status tqr_generate_guide(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len) {
+    if (!rates || ndev < 1 || !len) return fail(nullptr, TQR_ERR_ARG, "generate_guide: bad arguments");
+    std::vector<int32_t> r(rates, rates + ndev);
+    for (int x : r) if (x <= 0) return fail(nullptr, TQR_ERR_ARG, "generate_guide: rates must be > 0");
+    auto ga = generate_guide(r);
+    *len = (int32_t)ga.size();
+    if (guide) {
+        if (cap < (int32_t)ga.size()) return fail(nullptr, TQR_ERR_ARG, "generate_guide: capacity %d < %zu", cap, ga.size());
+        std::copy(ga.begin(), ga.end(), guide);
+    }
+    return TQR_OK;
+}
+
+static tqr_status validate_guide(int32_t ndev, const int32_t* guide, int32_t guide_len, std::vector<int32_t>& g) {
+    if (!guide) {
+        g.resize(ndev);
+        for (int d = 0; d < ndev; ++d) g[d] = d;
+        return TQR_OK;
+    }
+    if (guide_len < 1) return fail(nullptr, TQR_ERR_ARG, "guide_len must be >= 1");
+    g.assign(guide, guide + guide_len);
+    for (int v : g) if (v < 0 || v >= ndev) return fail(nullptr, TQR_ERR_ARG, "guide entry %d outside [0, %d)", v, ndev);
+    return TQR_OK;
+}
+
+tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const int32_t* guide, int32_t guide_len,
+                        int32_t rank, int32_t* ops, int64_t cap, int64_t* count) {
+    if (m < 1 || n < 1 || m < n || nb < 1 || n % nb || m % nb || ndev < 1 || rank < 0 || rank >= ndev || !count)
+        return fail(nullptr, TQR_ERR_ARG, "schedule: bad arguments");
+    std::vector<int32_t> g;
+    tqr_status st = validate_guide(ndev, guide, guide_len, g);
+    if (st) return st;
+    const int64_t q = n / nb;
+    std::vector<int32_t> owner_of(q);
+    for (int64_t j = 0; j < q; ++j) owner_of[j] = g[j % g.size()];
+    std::vector<int32_t> out;
+    build_schedule(q, owner_of, rank, out);
+    *count = (int64_t)out.size() / 5;
+    if (ops) {
+        if (cap < *count) return fail(nullptr, TQR_ERR_ARG, "schedule: capacity %lld < %lld", (long long)cap, (long long)*count);
+        std::copy(out.begin(), out.end(), ops);
+    }
+    return TQR_OK;
+}
+
+tqr_status tqr_nccl_unique_id(void* id128) {
+    if (!id128) return fail(nullptr, TQR_ERR_ARG, "nccl_unique_id: NULL");
+    const char* why = nullptr;
+    const tqr::NcclApi* api = tqr::nccl_api(&why);
+    if (!api) return fail(nullptr, TQR_ERR_NCCL, "NCCL unavailable: %s", why);
+    ncclUniqueId id;
+    if (api->GetUniqueId(&id) != ncclSuccess) return fail(nullptr, TQR_ERR_NCCL, "ncclGetUniqueId failed");
+    std::memcpy(id128, &id, sizeof(id));
+    return TQR_OK;
+}
+
+tqr_status tqr_create(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
+                      const int32_t* guide, int32_t guide_len, tqr_plan* out) {
+    return tqr_create_ex(m, n, nb, ib, dtype, ndev, guide, guide_len, nullptr, out);
+}
+
+tqr_status tqr_destroy(tqr_plan h) {
+    if (!h) return TQR_OK;
+    for (auto& o : h->owners) {
+        cudaSetDevice(o.dev);
+        if (o.s_panel) cudaStreamSynchronize(o.s_panel);
+        if (o.s_upd) cudaStreamSynchronize(o.s_upd);
+        if (o.s_comm) cudaStreamSynchronize(o.s_comm);
+    }
+    if (h->comm && h->nccl) h->nccl->CommDestroy(h->comm);
+    if (!h->owners.empty()) cudaSetDevice(h->owners[0].dev);
+    if (h->bw) cudaFree(h->bw);
+    if (h->rcm) cudaFree(h->rcm);
+    if (h->dflag) cudaFree(h->dflag);
+    for (auto& o : h->owners) free_owner(o);
+    cudaGetLastError();
+    delete h;
+    return TQR_OK;
+}
+
+tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
+                         const int32_t* guide, int32_t guide_len, const tqr_options* opt, tqr_plan* out) {
+    if (!out) return fail(nullptr, TQR_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (m < 1 || n < 1 || m < n) return fail(nullptr, TQR_ERR_ARG, "need m >= n >= 1 (m=%lld n=%lld)", (long long)m, (long long)n);
+    if (nb < 1 || ib < 1 || ib > nb || nb % ib) return fail(nullptr, TQR_ERR_ARG, "need 1 <= ib <= nb, nb %% ib == 0");
+    if (dtype != TQR_F64 && dtype != TQR_F32) return fail(nullptr, TQR_ERR_ARG, "unknown dtype");
+    if (ndev < 1) return fail(nullptr, TQR_ERR_ARG, "ndev must be >= 1");
+    std::vector<int32_t> g;
+    tqr_status st = validate_guide(ndev, guide, guide_len, g);
+    if (st) return st;
+    if (m % nb || n % nb) return fail(nullptr, TQR_ERR_UNSUPPORTED, "m and n must be multiples of nb in this build");
+    if (!supported_nb_ib(nb, ib)) return fail(nullptr, TQR_ERR_UNSUPPORTED, "nb in {64,128,256,512}, ib in {16,32} only");
+    if (dtype != TQR_F64) return fail(nullptr, TQR_ERR_UNSUPPORTED, "FP32 path not in this build");
+    tqr_options o{};
+    if (opt) o = *opt;
+    const int world = o.world > 1 ? o.world : 1;
+    if (world > 1 && (o.rank < 0 || o.rank >= world || ndev != world || !o.nccl_id))
+        return fail(nullptr, TQR_ERR_ARG, "multi-process: need 0 <= rank < world == ndev and nccl_id");
+    int ndevices = 0;
+    if (cudaGetDeviceCount(&ndevices) != cudaSuccess || ndevices < 1) {
+        cudaGetLastError();
+        return fail(nullptr, TQR_ERR_CUDA, "no CUDA device");
+    }
+    if (world == 1 && !o.logical_devices && ndev > ndevices)
+        return fail(nullptr, TQR_ERR_ARG, "ndev %d > %d visible CUDA devices (set logical_devices)", ndev, ndevices);
+
+    tqr_plan h = new tqr_plan_s();
+    h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)(m / nb); h->q = (int)(n / nb);
+    h->dtype = dtype; h->ndev = ndev; h->guide = g;
+    h->logical = o.logical_devices != 0;
+    h->rank = world > 1 ? o.rank : 0;
+    h->world = world;
+    h->lookahead = o.no_lookahead == 0;
+    h->profile = o.profile != 0;
+    h->owner_of.resize(h->q);
+    for (int j = 0; j < h->q; ++j) h->owner_of[j] = g[j % g.size()];
+
+    int cur = 0;
+    cudaGetDevice(&cur);
+    const int nown = world > 1 ? 1 : ndev;
+    h->owners.resize(nown);
+    auto bail = [&](tqr_status s) { std::string e = h->err; tqr_destroy(h); g_create_error = e; return s; };
+    int prio_lo = 0, prio_hi = 0;
+    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    const int64_t p = h->p, tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb;
+    for (int li = 0; li < nown; ++li) {
+        Owner& ow = h->owners[li];
+        ow.id = world > 1 ? h->rank : li;
+        ow.dev = (world > 1 || h->logical) ? cur : li;
+        ow.lidx.assign(h->q, -1);
+        for (int j = 0; j < h->q; ++j)
+            if (h->owner_of[j] == ow.id) { ow.lidx[j] = (int32_t)ow.cols.size(); ow.cols.push_back(j); }
+        if (cudaSetDevice(ow.dev) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "cudaSetDevice(%d)", ow.dev));
+        auto mk = [&](cudaStream_t* s, int prio) { return cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, prio); };
+        if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi))
+            return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
+        for (auto* v : {&ow.ev_panel, &ow.ev_recv, &ow.ev_upd, &ow.ev_look}) {
+            v->assign(h->q, nullptr);
+            for (auto& e : *v)
+                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                    return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
+        }
+        if (h->profile) {
+            for (auto* v : {&ow.tm0, &ow.tm1, &ow.tp0, &ow.tp1}) {
+                v->assign(h->q, nullptr);
+                for (auto& e : *v)
+                    if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
+            }
+            ow.tm_used.assign(h->q, 0);
+            ow.tp_used.assign(h->q, 0);
+        }
+        const size_t nc = ow.cols.size();
+        auto alloc = [&](double** ptr, size_t elems) -> bool {
+            if (elems == 0) return true;
+            if (cudaMalloc(ptr, elems * sizeof(double)) != cudaSuccess) { cudaGetLastError(); return false; }
+            return true;
+        };
+        if (!alloc(&ow.tiles, nc * p * tile) || !alloc(&ow.T, nc * p * tsz) || !alloc(&ow.Vexp, nc * tile))
+            return bail(fail(h, TQR_ERR_ALLOC, "tile storage allocation failed"));
+        if (nc) {
+            if (cudaMemset(ow.T, 0, nc * p * tsz * sizeof(double)) != cudaSuccess)
+                return bail(fail(h, TQR_ERR_CUDA, "memset"));
+            if (cudaMalloc(&ow.cols_dev, nc * sizeof(int32_t)) != cudaSuccess ||
+                cudaMemcpy(ow.cols_dev, ow.cols.data(), nc * sizeof(int32_t), cudaMemcpyHostToDevice) != cudaSuccess)
+                return bail(fail(h, TQR_ERR_ALLOC, "cols allocation failed"));
+        }
+        // receive slots are needed when some remote panel k precedes an owned column
+        bool need_rb = world > 1;   // every rank takes part in every ncclBroadcast
+        for (int k = 0; k < h->q && !need_rb; ++k)
+            if (h->owner_of[k] != ow.id)
+                for (int j = k + 1; j < h->q; ++j) if (h->owner_of[j] == ow.id) { need_rb = true; break; }
+        if (need_rb)
+            for (int s = 0; s < 2; ++s)
+                if (!alloc(&ow.rb_tiles[s], p * tile) || !alloc(&ow.rb_T[s], p * tsz) || !alloc(&ow.rb_V[s], tile))
+                    return bail(fail(h, TQR_ERR_ALLOC, "receive buffer allocation failed"));
+        if (nc) {
+            const size_t nfl = (size_t)p * (nb / ib);
+            if (cudaMalloc(&ow.flags, nfl * sizeof(unsigned)) != cudaSuccess ||
+                cudaMemset(ow.flags, 0, nfl * sizeof(unsigned)) != cudaSuccess)
+                return bail(fail(h, TQR_ERR_ALLOC, "flag allocation failed"));
+        }
+    }
+    // peer access between physical owners (single-process, several GPUs)
+    if (world == 1 && !h->logical && ndev > 1) {
+        for (int a = 0; a < ndev; ++a)
+            for (int b = 0; b < ndev; ++b) {
+                if (a == b) continue;
+                int can = 0;
+                cudaDeviceCanAccessPeer(&can, a, b);
+                if (can) { cudaSetDevice(a); cudaDeviceEnablePeerAccess(b, 0); cudaGetLastError(); }
+            }
+    }
+    if (world > 1) {
+        const char* why = nullptr;
+        h->nccl = tqr::nccl_api(&why);
+        if (!h->nccl) return bail(fail(h, TQR_ERR_NCCL, "NCCL unavailable: %s", why));
+        ncclUniqueId id;
+        std::memcpy(&id, o.nccl_id, sizeof(id));
+        cudaSetDevice(cur);
+        ncclResult_t r = h->nccl->CommInitRank(&h->comm, world, id, h->rank);
+        if (r != ncclSuccess) return bail(fail(h, TQR_ERR_NCCL, "ncclCommInitRank: %s", h->nccl->GetErrorString(r)));
+    }
+    cudaSetDevice(cur);
+    *out = h;
+    return TQR_OK;
+}
+
+int32_t tqr_owner(tqr_plan h, int64_t j) {
+    if (!h || j < 0 || j >= h->q) return -1;
+    return h->owner_of[j];
+}
+
+int64_t tqr_launch_count(tqr_plan h) {
+    if (!h) return 0;
+    int64_t c = h->launches;
+    h->launches = 0;
+    return c;
+}
+
+tqr_status tqr_kernel_stats(tqr_plan h, int32_t which, int64_t* count, double* ms, double* flops, int32_t reset) {
+    if (!h || which < 0 || which > 3) return fail(h, TQR_ERR_ARG, "kernel_stats: bad arguments");
+    if (count) *count = h->stats[which].count;
+    if (ms) *ms = h->stats[which].ms;
+    if (flops) *flops = h->stats[which].flops;
+    if (reset) h->stats[which] = KStat();
+    return TQR_OK;
+}
+
+// ------------------------------------------------------------------ a1: load
+tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
+    if (!h) return TQR_ERR_ARG;
+    if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (!Av || lda < h->m) return fail(h, TQR_ERR_ARG, "load: A is NULL or lda < m");
+    const double* A = static_cast<const double*>(Av);
+    const PtrInfo pi = classify(A);
+    const int64_t p = h->p, nb = h->nb, tile = nb * nb;
+    h->factored = false;
+    for (auto& o : h->owners) {
+        if (o.cols.empty()) continue;
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        const int nc = (int)o.cols.size();
+        if (pi.kind == Mem::Device && pi.dev == o.dev) {
+            CUDA_TRY(h, tqr::launch_to_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, nc, p * tile, (int)nb, (int)p, o.s_upd));
+            h->launches++;
+        } else {
+            tqr_status st = ensure_io(h, o);
+            if (st) return st;
+            for (int lc = 0; lc < nc; ++lc) {
+                const int64_t j = o.cols[lc];
+                CUDA_TRY(h, cudaMemcpy2DAsync(o.io + (int64_t)lc * h->m * nb, h->m * sizeof(double),
+                                              A + j * nb * lda, lda * sizeof(double), h->m * sizeof(double), nb,
+                                              cudaMemcpyDefault, o.s_upd));
+            }
+            // io holds the owned columns in local order: group lc at io + lc*m*nb -> use an identity map
+            CUDA_TRY(h, tqr::launch_to_tiles(o.io, h->m, h->m * nb, o.tiles, nullptr, nc, p * tile, (int)nb, (int)p, o.s_upd));
+            h->launches++;
+        }
+    }
+    return sync_all(h);
+}
+
+// ------------------------------------------------------------------ a2-a7: factor
+tqr_status tqr_factor_tiles(tqr_plan h) {
+    if (!h) return TQR_ERR_ARG;
+    if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
+    const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile;
+    const unsigned epoch0 = h->epoch;
+    h->epoch += (unsigned)q + 1;
+    // order all owner streams after whatever ran before (load, previous calls)
+    for (auto& o : h->owners) {
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        CUDA_TRY(h, cudaStreamSynchronize(o.s_upd));
+        if (h->profile) { std::fill(o.tm_used.begin(), o.tm_used.end(), 0); std::fill(o.tp_used.begin(), o.tp_used.end(), 0); }
+    }
+    for (int k = 0; k < q; ++k) {
+        const int ok = h->owner_of[k];
+        Owner* O = h->local(ok);
+        // ---- PANEL(k)
+        if (O) {
+            CUDA_TRY(h, cudaSetDevice(O->dev));
+            if (k > 0 && !h->lookahead) CUDA_TRY(h, cudaStreamWaitEvent(O->s_panel, O->ev_upd[k - 1], 0));
+            const int lc = O->lidx[k];
+            PanelArgs a;
+            a.col = O->tiles + lc * colsz;
+            a.T = O->T + lc * (int64_t)p * tsz;
+            a.Vexp = O->Vexp + lc * tile;
+            a.flags = O->flags;
+            a.epoch = epoch0 + (unsigned)k + 1;
+            a.k = k;
+            a.p = p;
+            if (h->profile) CUDA_TRY(h, cudaEventRecord(O->tp0[k], O->s_panel));
+            CUDA_TRY(h, tqr::launch_panel(nb, ib, a, O->s_panel));
+            h->launches++;
+            if (h->profile) { CUDA_TRY(h, cudaEventRecord(O->tp1[k], O->s_panel)); O->tp_used[k] = 1; }
+            CUDA_TRY(h, cudaEventRecord(O->ev_panel[k], O->s_panel));
+        }
+        // ---- BCAST(k): the reflector tiles k..p-1, their T factors and the explicit V
+        if (h->multiproc()) {
+            Owner& R = h->owners[0];
+            CUDA_TRY(h, cudaSetDevice(R.dev));
+            const int slot = k & 1;
+            const bool root = (ok == h->rank);
+            if (root) CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_panel[k], 0));
+            if (!root && k >= 2) {
+                CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_upd[k - 2], 0));
+                CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
+            }
+            double *bt, *bT, *bV;
+            if (root) {
+                const int lc = R.lidx[k];
+                bt = R.tiles + lc * colsz; bT = R.T + lc * (int64_t)p * tsz; bV = R.Vexp + lc * tile;
+            } else {
+                bt = R.rb_tiles[slot]; bT = R.rb_T[slot]; bV = R.rb_V[slot];
+            }
+            const bool need = root || bt != nullptr;
+            double dummy_needed = 0; (void)dummy_needed;
+            if (need) {
+                NCCL_TRY(h, h->nccl->GroupStart());
+                NCCL_TRY(h, h->nccl->Broadcast(bt + k * tile, bt + k * tile, (size_t)(p - k) * tile, ncclFloat64, ok, h->comm, R.s_comm));
+                NCCL_TRY(h, h->nccl->Broadcast(bT + k * tsz, bT + k * tsz, (size_t)(p - k) * tsz, ncclFloat64, ok, h->comm, R.s_comm));
+                NCCL_TRY(h, h->nccl->Broadcast(bV, bV, (size_t)tile, ncclFloat64, ok, h->comm, R.s_comm));
+                NCCL_TRY(h, h->nccl->GroupEnd());
+            }
+            CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
+        } else {
+            for (auto& D : h->owners) {
+                if (D.id == ok) continue;
+                bool needs = false;
+                for (int32_t j : D.cols) if (j > k) { needs = true; break; }
+                if (!needs) continue;
+                CUDA_TRY(h, cudaSetDevice(D.dev));
+                const int slot = k & 1;
+                CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_panel[k], 0));
+                if (k >= 2) {
+                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_upd[k - 2], 0));
+                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_look[k - 2], 0));
+                }
+                const int lc = O->lidx[k];
+                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_tiles[slot] + k * tile, D.dev, O->tiles + lc * colsz + k * tile,
+                                                O->dev, sizeof(double) * (size_t)(p - k) * tile, D.s_comm));
+                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_T[slot] + k * tsz, D.dev, O->T + lc * (int64_t)p * tsz + k * tsz,
+                                                O->dev, sizeof(double) * (size_t)(p - k) * tsz, D.s_comm));
+                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, O->Vexp + lc * tile, O->dev,
+                                                sizeof(double) * (size_t)tile, D.s_comm));
+                CUDA_TRY(h, cudaEventRecord(D.ev_recv[k], D.s_comm));
+            }
+        }
+        // ---- UPDATE(k) on every local owner
+        for (auto& D : h->owners) {
+            CUDA_TRY(h, cudaSetDevice(D.dev));
+            const bool mine = (D.id == ok);
+            UpdateArgs u;
+            if (mine) {
+                const int lc = D.lidx[k];
+                u.V = D.tiles + lc * colsz; u.T = D.T + lc * (int64_t)p * tsz; u.Vexp = D.Vexp + lc * tile;
+            } else {
+                const int slot = k & 1;
+                u.V = D.rb_tiles[slot]; u.T = D.rb_T[slot]; u.Vexp = D.rb_V[slot];
+            }
+            u.X = D.tiles; u.col_stride = colsz; u.tile_stride = tile; u.ld = nb;
+            u.k = k; u.p = p; u.do_unmqr = 1;
+            cudaEvent_t ready = mine ? D.ev_panel[k] : D.ev_recv[k];
+            // local columns j > k form a suffix of D.cols
+            int first = (int)(std::upper_bound(D.cols.begin(), D.cols.end(), k) - D.cols.begin());
+            int ncols = (int)D.cols.size() - first;
+            const bool la = h->lookahead && ncols > 0 && D.cols[first] == k + 1;
+            if (la) {
+                CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, ready, 0));
+                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_upd[k - 1], 0));
+                u.group0 = first;
+                CUDA_TRY(h, tqr::launch_update(nb, ib, w_look(h), u, nb / w_look(h), true, D.s_panel));
+                h->launches++;
+                first += 1;
+                ncols -= 1;
+            }
+            CUDA_TRY(h, cudaEventRecord(D.ev_look[k], D.s_panel));
+            CUDA_TRY(h, cudaStreamWaitEvent(D.s_upd, ready, 0));
+            if (ncols > 0) {
+                u.group0 = first;
+                if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[k], D.s_upd));
+                CUDA_TRY(h, tqr::launch_update(nb, ib, w_bulk(h), u, ncols * (nb / w_bulk(h)), true, D.s_upd));
+                h->launches++;
+                if (h->profile) {
+                    CUDA_TRY(h, cudaEventRecord(D.tm1[k], D.s_upd));
+                    D.tm_used[k] = 1;
+                    h->stats[0].flops += flops_update(h, k, ncols);
+                    h->stats[0].count += 1;
+                }
+            }
+            CUDA_TRY(h, cudaEventRecord(D.ev_upd[k], D.s_upd));
+        }
+    }
+    tqr_status st = sync_all(h);
+    if (st) return st;
+    if (h->profile) {
+        for (auto& o : h->owners) {
+            CUDA_TRY(h, cudaSetDevice(o.dev));
+            for (int k = 0; k < q; ++k) {
+                float ms = 0.f;
+                if (o.tm_used[k]) { CUDA_TRY(h, cudaEventElapsedTime(&ms, o.tm0[k], o.tm1[k])); h->stats[0].ms += ms; }
+                if (o.tp_used[k]) {
+                    CUDA_TRY(h, cudaEventElapsedTime(&ms, o.tp0[k], o.tp1[k]));
+                    h->stats[1].ms += ms; h->stats[1].count += 1; h->stats[1].flops += flops_panel(h, k);
+                }
+            }
+        }
+    }
+    h->factored = true;
+    return TQR_OK;
+}
+
+// ------------------------------------------------------------------ a8: R out
+tqr_status tqr_store_r(tqr_plan h, void* Av, int64_t lda) {
+    if (!h) return TQR_ERR_ARG;
+    if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (!h->factored) return fail(h, TQR_ERR_STATE, "store_r before factor");
+    if (!Av || lda < h->m) return fail(h, TQR_ERR_ARG, "store_r: A is NULL or lda < m");
+    double* A = static_cast<double*>(Av);
+    const PtrInfo pi = classify(A);
+    const int64_t p = h->p, nb = h->nb, tile = nb * nb;
+    for (auto& o : h->owners) {
+        if (o.cols.empty()) continue;
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        const int nc = (int)o.cols.size();
+        if (pi.kind == Mem::Device && pi.dev == o.dev) {
+            CUDA_TRY(h, tqr::launch_from_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, nc, p * tile, (int)nb, (int)p, h->m, 0, o.s_upd));
+            h->launches++;
+        } else {
+            tqr_status st = ensure_io(h, o);
+            if (st) return st;
+            CUDA_TRY(h, tqr::launch_from_tiles(o.io, h->m, h->m * nb, o.tiles, o.cols_dev, nc, p * tile, (int)nb, (int)p, h->m, 1, o.s_upd));
+            h->launches++;
+            for (int lc = 0; lc < nc; ++lc) {
+                const int64_t j = o.cols[lc];
+                CUDA_TRY(h, cudaMemcpy2DAsync(A + j * nb * lda, lda * sizeof(double), o.io + (int64_t)lc * h->m * nb,
+                                              h->m * sizeof(double), h->m * sizeof(double), nb, cudaMemcpyDefault, o.s_upd));
+            }
+        }
+    }
+    return sync_all(h);
+}
+
+tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
+    tqr_status st = tqr_load(h, A, lda);
+    if (st) return st;
+    st = tqr_factor_tiles(h);
+    if (st) return st;
+    return tqr_store_r(h, A, lda);
+}
+
+// ------------------------------------------------------------------ apply Q^T / Q, solve
+static tqr_status single_device(tqr_plan h, int* dev) {
+    if (h->multiproc()) return fail(h, TQR_ERR_UNSUPPORTED, "apply/solve: multi-process plans not supported in this build");
+    *dev = h->owners[0].dev;
+    for (auto& o : h->owners)
+        if (o.dev != *dev) return fail(h, TQR_ERR_UNSUPPORTED, "apply/solve: owners on several GPUs not supported in this build");
+    return TQR_OK;
+}
+
+static tqr_status apply_device(tqr_plan h, char trans, double* Bw, int64_t ldw, int64_t nslices, cudaStream_t s) {
+    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
+    const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile;
+    const bool fwd = (trans == 'T' || trans == 't');
+    for (int s_ = 0; s_ < q; ++s_) {
+        const int k = fwd ? s_ : q - 1 - s_;
+        Owner* O = h->local(h->owner_of[k]);
+        const int lc = O->lidx[k];
+        UpdateArgs u;
+        u.V = O->tiles + lc * colsz; u.T = O->T + lc * (int64_t)p * tsz; u.Vexp = O->Vexp + lc * tile;
+        u.X = Bw; u.col_stride = (int64_t)nb * ldw; u.tile_stride = nb; u.ld = ldw;
+        u.group0 = 0; u.k = k; u.p = p; u.do_unmqr = 1;
+        CUDA_TRY(h, tqr::launch_update(nb, ib, 32, u, (int)nslices, fwd, s));
+        h->launches++;
+    }
+    return TQR_OK;
+}
+
+static tqr_status stage_b(tqr_plan h, const double* B, int64_t ldb, int64_t nrhs, int64_t* nslices, cudaStream_t s) {
+    const int64_t pad = (nrhs + 31) / 32 * 32;
+    *nslices = pad / 32;
+    const size_t need = (size_t)h->m * pad;
+    if (need > h->bw_elems) {
+        if (h->bw) cudaFree(h->bw);
+        h->bw = nullptr;
+        h->bw_elems = 0;
+        CUDA_TRY(h, cudaMalloc(&h->bw, need * sizeof(double)));
+        h->bw_elems = need;
+    }
+    CUDA_TRY(h, cudaMemsetAsync(h->bw, 0, need * sizeof(double), s));
+    CUDA_TRY(h, cudaMemcpy2DAsync(h->bw, h->m * sizeof(double), B, ldb * sizeof(double), h->m * sizeof(double), nrhs,
+                                  cudaMemcpyDefault, s));
+    return TQR_OK;
+}
+
+tqr_status tqr_apply_qt(tqr_plan h, char trans, void* Bv, int64_t ldb, int64_t nrhs) {
+    if (!h) return TQR_ERR_ARG;
+    if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (!h->factored) return fail(h, TQR_ERR_STATE, "apply_qt before a successful factor");
+    if (!(trans == 'T' || trans == 't' || trans == 'N' || trans == 'n')) return fail(h, TQR_ERR_ARG, "trans must be 'T' or 'N'");
+    if (nrhs < 0 || (nrhs > 0 && (!Bv || ldb < h->m))) return fail(h, TQR_ERR_ARG, "apply_qt: bad B/ldb/nrhs");
+    if (nrhs == 0) return TQR_OK;
+    int dev = 0;
+    tqr_status st = single_device(h, &dev);
+    if (st) return st;
+    CUDA_TRY(h, cudaSetDevice(dev));
+    cudaStream_t s = h->owners[0].s_upd;
+    double* B = static_cast<double*>(Bv);
+    int64_t nsl = 0;
+    st = stage_b(h, B, ldb, nrhs, &nsl, s);
+    if (st) return st;
+    st = apply_device(h, trans, h->bw, h->m, nsl, s);
+    if (st) return st;
+    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, h->m * sizeof(double), h->m * sizeof(double), nrhs,
+                                  cudaMemcpyDefault, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    return TQR_OK;
+}
+
+tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
+    if (!h) return TQR_ERR_ARG;
+    if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (!h->factored) return fail(h, TQR_ERR_STATE, "solve_ls before a successful factor");
+    if (nrhs < 0 || (nrhs > 0 && (!Bv || ldb < h->m))) return fail(h, TQR_ERR_ARG, "solve_ls: bad B/ldb/nrhs");
+    if (nrhs == 0) return TQR_OK;
+    int dev = 0;
+    tqr_status st = single_device(h, &dev);
+    if (st) return st;
+    CUDA_TRY(h, cudaSetDevice(dev));
+    cudaStream_t s = h->owners[0].s_upd;
+    double* B = static_cast<double*>(Bv);
+    int64_t nsl = 0;
+    st = stage_b(h, B, ldb, nrhs, &nsl, s);
+    if (st) return st;
+    st = apply_device(h, 'T', h->bw, h->m, nsl, s);
+    if (st) return st;
+    // gather R (n x n, column-major) from every owner
+    const int64_t n = h->n, nb = h->nb, tile = nb * nb;
+    if (!h->rcm) CUDA_TRY(h, cudaMalloc(&h->rcm, sizeof(double) * (size_t)n * n));
+    if (!h->dflag) CUDA_TRY(h, cudaMalloc(&h->dflag, sizeof(int64_t)));
+    for (auto& o : h->owners) {
+        if (o.cols.empty()) continue;
+        CUDA_TRY(h, tqr::launch_from_tiles(h->rcm, n, nb * n, o.tiles, o.cols_dev, (int)o.cols.size(), h->p * tile,
+                                           (int)nb, h->p, n, 0, s));
+        h->launches++;
+    }
+    const int64_t big = INT64_MAX;
+    CUDA_TRY(h, cudaMemcpyAsync(h->dflag, &big, sizeof(int64_t), cudaMemcpyHostToDevice, s));
+    CUDA_TRY(h, tqr::launch_zero_diag_check(h->rcm, n, n, h->dflag, s));
+    int64_t first_zero = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(&first_zero, h->dflag, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    if (first_zero != big) return fail(h, TQR_ERR_SINGULAR, "R(%lld,%lld) == 0", (long long)first_zero, (long long)first_zero);
+    CUDA_TRY(h, tqr::launch_trsv_upper(h->rcm, n, h->bw, h->m, n, nrhs, s));
+    h->launches++;
+    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, h->m * sizeof(double), n * sizeof(double), nrhs,
+                                  cudaMemcpyDefault, s));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    return TQR_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------ NCCL loader
+namespace tqr {
+const NcclApi* nccl_api(const char** why) {
+    static NcclApi api;
+    static bool tried = false;
+    static const char* reason = "not loaded";
+    if (!tried) {
+        tried = true;
+        void* lib = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!lib) lib = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!lib) {
+            reason = "dlopen(libnccl.so.2) failed";
+        } else {
+            bool ok = true;
+            auto sym = [&](const char* n) { void* s = dlsym(lib, n); if (!s) ok = false; return s; };
+            api.GetUniqueId = (decltype(api.GetUniqueId))sym("ncclGetUniqueId");
+            api.CommInitRank = (decltype(api.CommInitRank))sym("ncclCommInitRank");
+            api.CommDestroy = (decltype(api.CommDestroy))sym("ncclCommDestroy");
+            api.CommGetAsyncError = (decltype(api.CommGetAsyncError))sym("ncclCommGetAsyncError");
+            api.Broadcast = (decltype(api.Broadcast))sym("ncclBroadcast");
+            api.GroupStart = (decltype(api.GroupStart))sym("ncclGroupStart");
+            api.GroupEnd = (decltype(api.GroupEnd))sym("ncclGroupEnd");
+            api.GetErrorString = (decltype(api.GetErrorString))sym("ncclGetErrorString");
+            api.ok = ok;
+            if (!ok) reason = "libnccl.so.2 lacks a required symbol";
+        }
+    }
+    if (!api.ok) { if (why) *why = reason; return nullptr; }
+    return &api;
+}
+}  // namespace tqr

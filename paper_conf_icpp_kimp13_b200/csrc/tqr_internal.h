@@ -1,0 +1,55 @@
+// tqr_internal.h -- kernel argument blocks and launchers shared by the host runtime (tqr_api.cpp)
+// and the sm_100a kernels (kernels/qr_kernels.cu).  Not part of the public ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace tqr {
+
+// Panel step k on the owner of column k: GEQRT(k,k) + TSQRT(i,k), i = k+1..p-1.
+struct PanelArgs {
+    double* col;       // the owner's tiles of column k: tile i at col + i*nb*nb (column-major nb x nb)
+    double* T;         // T factors of column k: tile i at T + i*ib*nb (ib x nb, LAPACK dgeqrt layout)
+    double* Vexp;      // explicit unit-lower V of the diagonal tile (nb x nb), written by GEQRT
+    unsigned* flags;   // p * (nb/ib) publication flags
+    unsigned epoch;    // value published for this launch (monotone across launches)
+    int k;             // step (tile column / diagonal tile row)
+    int p;             // number of row tiles
+};
+
+// Trailing update of step k over `ngroups` column groups (UNMQR + TSMQR chain), or the
+// application of panel k's Q^T / Q to a right-hand side block (tqr_apply_qt).
+struct UpdateArgs {
+    const double* V;     // reflector tiles of panel k: tile i at V + i*nb*nb (rows k+1.. used)
+    const double* Vexp;  // explicit V of the diagonal tile
+    const double* T;     // T factors: tile i at T + i*ib*nb
+    double* X;           // target: element (tile i, r, c) of group gidx at
+                         //   X + gidx*col_stride + i*tile_stride + c*ld + r
+    int64_t col_stride;
+    int64_t tile_stride;
+    int64_t ld;
+    int group0;          // first group index
+    int k, p;
+    int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
+};
+
+cudaError_t launch_panel(int nb, int ib, const PanelArgs& a, cudaStream_t s);
+// nslices CTAs; CTA b works on columns [b*w, b*w + w) counted from group0 (groups are nb wide)
+cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslices, bool trans, cudaStream_t s);
+// src column group of local column lc at src + (cols_dev ? cols[lc] : lc)*src_group_stride (ld = lda)
+// -> tiles at dst + lc*dst_col_stride
+cudaError_t launch_to_tiles(const double* src, int64_t lda, int64_t src_group_stride, double* dst,
+                            const int32_t* cols_dev, int ncols, int64_t dst_col_stride, int nb, int p,
+                            cudaStream_t s);
+// tiles -> column-major rows [0, m_rows) with zeros below the diagonal (global column of local
+// column lc is cols[lc]); destination group at dst + (local_dst ? lc : cols[lc])*dst_group_stride
+cudaError_t launch_from_tiles(double* dst, int64_t lda, int64_t dst_group_stride, const double* src,
+                              const int32_t* cols_dev, int ncols, int64_t src_col_stride, int nb, int p,
+                              int64_t m_rows, int local_dst, cudaStream_t s);
+cudaError_t launch_trsv_upper(const double* R, int64_t ldr, double* C, int64_t ldc, int64_t n, int64_t nrhs,
+                              cudaStream_t s);
+cudaError_t launch_zero_diag_check(const double* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s);
+size_t panel_smem_bytes(int nb, int ib);
+size_t update_smem_bytes(int nb, int ib, int w);
+
+}  // namespace tqr

@@ -1,0 +1,99 @@
+"""CPU-only checks of the C-ABI library: it loads, exports every symbol include/tqr.h
+declares, and its pure host logic (guide array, schedule, argument validation) is right.
+No compute calls are made here (no GPU in this container)."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_icpp_kimp13_b200 as tqr
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    from paper_conf_icpp_kimp13_b200 import build
+    build.build()
+    return tqr.lib()
+
+
+def header_symbols():
+    src = open(os.path.join(ROOT, "include", "tqr.h")).read()
+    decl = r"^(?:tqr_status|const char\*|int32_t|int64_t)\s+(tqr_[a-z0-9_]+)\s*\("
+    return sorted(set(re.findall(decl, src, flags=re.M)))
+
+
+def test_header_symbols_exported(L):
+    syms = header_symbols()
+    assert "tqr_create" in syms and "tqr_solve_ls" in syms
+    for s in syms:
+        assert hasattr(L, s), s
+    assert sorted(syms) == sorted(tqr.EXPORTED)
+
+
+def test_status_strings(L):
+    for code in range(8):
+        assert L.tqr_status_string(code).decode().startswith(tqr.STATUS[code])
+
+
+def test_generate_guide_matches_oracle_and_paper(L):
+    assert tqr.tqr_generate_guide([8, 12, 4]) == [1, 0, 1, 0, 1, 2]
+    rng = np.random.default_rng(1)
+    for _ in range(100):
+        rates = [int(x) for x in rng.integers(1, 9, size=int(rng.integers(1, 9)))]
+        assert tqr.tqr_generate_guide(rates) == oracle.guide.generate_array(oracle.guide.get_ratio(rates))
+
+
+def _expected_schedule(q, guide, rank):
+    own = [oracle.guide.distribute(j, guide) for j in range(q)]
+    out = []
+    for k in range(q):
+        if own[k] == rank:
+            out.append((0, k, k, k, own[k]))
+        out.append((1, k, k, k, own[k]))
+        out += [(2, k, k, j, own[k]) for j in range(k + 1, q) if own[j] == rank]
+    return out
+
+
+@pytest.mark.parametrize("guide,ndev", [([0, 1], 2), ([1, 0, 1, 0, 1, 2], 3), ([0], 1), ([3, 2, 1, 0], 4)])
+def test_schedule_covers_dag(L, guide, ndev):
+    m, n, nb = 1024, 768, 64
+    q = n // nb
+    per_rank = [tqr.tqr_schedule(m, n, nb, ndev, guide, r) for r in range(ndev)]
+    for r in range(ndev):
+        assert per_rank[r] == _expected_schedule(q, guide, r)
+    # union: every panel once, every update (k, j>k) exactly once, on the owner of j (Eq. 12)
+    panels = [op for ops in per_rank for op in ops if op[0] == 0]
+    assert sorted(op[1] for op in panels) == list(range(q))
+    ups = sorted((op[1], op[3]) for ops in per_rank for op in ops if op[0] == 2)
+    assert ups == [(k, j) for k in range(q) for j in range(k + 1, q)]
+    # Table I (TS reading, Q6): per step k, 1 GEQRT, p-k-1 TSQRT, q-k-1 UNMQR, (p-k-1)(q-k-1) TSMQR
+    p = m // nb
+    for k in range(q):
+        n_up = sum(1 for (kk, j) in ups if kk == k)
+        assert n_up == q - k - 1
+        assert (p - k - 1) * n_up == (p - k - 1) * (q - k - 1)
+
+
+def test_schedule_rejects_bad_args(L):
+    with pytest.raises(tqr.TqrError):
+        tqr.tqr_schedule(100, 64, 64, 1, None, 0)
+    with pytest.raises(tqr.TqrError):
+        tqr.tqr_schedule(128, 128, 64, 2, [0, 5], 0)
+
+
+def test_create_without_gpu_fails_cleanly(L):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(tqr.TqrError) as e:
+        tqr.Plan(128, 128, 64, 16)
+    assert e.value.status == 3
+    # argument errors are reported before any CUDA call
+    with pytest.raises(tqr.TqrError) as e:
+        tqr.Plan(64, 128, 64, 16)
+    assert e.value.status == 1
+    assert L.tqr_destroy(None) == 0
