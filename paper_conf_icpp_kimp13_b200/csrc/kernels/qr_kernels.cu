@@ -99,7 +99,7 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     constexpr int NBLK = NB / IB;
     const int grp = blockIdx.x / SPG;
     const int c0 = (blockIdx.x % SPG) * W;
-    double* Xg = a.X + (int64_t)(a.group0 + grp) * a.col_stride + (int64_t)c0 * a.ld;
+    double* Xg = a.X + (int64_t)(a.group0 + grp * a.gstride) * a.col_stride + (int64_t)c0 * a.ld;
     double* Xk = Xg + (int64_t)a.k * a.tile_stride;
     const int64_t vtile = (int64_t)NB * NB;
     Slice<NB, W, IB> X;

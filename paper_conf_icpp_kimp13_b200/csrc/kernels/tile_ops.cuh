@@ -93,32 +93,57 @@ struct Slice {
 };
 
 // V loads: the panel kernel reads V published by sibling CTAs of the same grid -> L2 (.cg);
-// the update kernel reads V that is immutable during the launch -> default path (L1-cached).
+// the update kernel reads V that is immutable during the launch -> read-only path (.nc).
 template <bool CG>
 __device__ __forceinline__ double2 vld2(const double* p) {
-    if constexpr (CG) return ld2_cg(p); else return ld2(p);
+    if constexpr (CG) return ld2_cg(p); else return __ldg(reinterpret_cast<const double2*>(p));
 }
 template <bool CG>
 __device__ __forceinline__ double vld(const double* p) {
-    if constexpr (CG) return ld_cg(p); else return *p;
+    if constexpr (CG) return ld_cg(p); else return __ldg(p);
 }
 
 // ---------------------------------------------------------------- apply one ib block
 // X (registers, NB x W) <- H_s X where H_s = I - V_s T_s^T V_s^T (TRANS) or I - V_s T_s V_s^T.
-//   Vs   : column s*IB of V (NB x IB, ld = ldv); rows < kmin are zero and skipped.
+//   Vs   : column s*IB of V (NB x IB, ld = ldv); rows < kmin are zero (their DMMAs skipped).
 //   Ts   : T block s (IB x IB column-major, ld = IB) = T_tile + s*IB*IB.
 //   top  : if non-null, the X1 rows (IB x W, element (r, c) at top[c*ldtop + r]).
-// Ends with no pending smem hazards for the caller except Wsm/red reuse (guarded inside).
+// Latency hiding (8 warps/SM only, 254 registers): every global operand is loaded one step
+// ahead of its use -- GEMM1's V fragments one row-fragment ahead, GEMM2's first fragments and
+// the top rows / T block before the reduction barriers, GEMM2's next k-step during the current.
 template <int NB, int W, int IB, bool TRANS, bool CG>
 __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>& sm,
                                             const double* __restrict__ Vs, int64_t ldv,
                                             const double* __restrict__ Ts,
                                             double* top, int64_t ldtop, int kmin) {
     using G = Geom<NB, W, IB>;
+    constexpr int NR = (W * IB + kThreads - 1) / kThreads;     // reduce outputs per thread
+    constexpr int NT = (IB * IB + kThreads - 1) / kThreads;    // T entries per thread
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW;
+    const int tid = threadIdx.x;
 
-    // ---- GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib)
+    // ---- (0) early loads: top rows and T block (consumed after the first barrier)
+    double topv[NR];
+#pragma unroll
+    for (int r = 0; r < NR; ++r) {
+        const int idx = tid + r * kThreads;
+        topv[r] = 0.0;
+        if (top && idx < W * IB) topv[r] = top[(int64_t)(idx / IB) * ldtop + (idx % IB)];
+    }
+    double tv[NT];
+#pragma unroll
+    for (int r = 0; r < NT; ++r) {
+        const int idx = tid + r * kThreads;
+        tv[r] = 0.0;
+        if (idx < IB * IB) {
+            const int rp = idx / IB, rr = idx % IB;
+            if constexpr (TRANS) { if (rp <= rr) tv[r] = vld<CG>(Ts + rr * IB + rp); }   // T(r', r): W' = T^T W
+            else                 { if (rp >= rr) tv[r] = vld<CG>(Ts + rp * IB + rr); }   // T(r, r'): W' = T W
+        }
+    }
+
+    // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib)
 #pragma unroll
     for (int jc = 0; jc < G::JF; jc += G::JC) {
         double c1[G::MF][G::JC][2];
@@ -126,20 +151,29 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
         for (int mf = 0; mf < G::MF; ++mf)
 #pragma unroll
             for (int j = 0; j < G::JC; ++j) c1[mf][j][0] = c1[mf][j][1] = 0.0;
+        const double* vb = Vs + (int64_t)(jc * 8 + g) * ldv + rbase + 2 * t;
+        double2 bn[G::JC];
+#pragma unroll
+        for (int j = 0; j < G::JC; ++j) bn[j] = vld2<CG>(vb + (int64_t)j * 8 * ldv);
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
-            if (rbase + nf * 8 + 8 <= kmin) continue;   // V rows all zero (warp-uniform)
             double2 b[G::JC];
 #pragma unroll
-            for (int j = 0; j < G::JC; ++j)
-                b[j] = vld2<CG>(Vs + (int64_t)((jc + j) * 8 + g) * ldv + rbase + nf * 8 + 2 * t);
+            for (int j = 0; j < G::JC; ++j) b[j] = bn[j];
+            if (nf + 1 < G::NF) {
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf)
+                for (int j = 0; j < G::JC; ++j) bn[j] = vld2<CG>(vb + (int64_t)j * 8 * ldv + (nf + 1) * 8);
+            }
+            if (rbase + nf * 8 + 8 > kmin) {                 // rows < kmin of V are zero
 #pragma unroll
-                for (int j = 0; j < G::JC; ++j) {
-                    dmma(c1[mf][j][0], c1[mf][j][1], X.acc[mf][nf][0], b[j].x);
-                    dmma(c1[mf][j][0], c1[mf][j][1], X.acc[mf][nf][1], b[j].y);
-                }
+                for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                    for (int j = 0; j < G::JC; ++j) dmma(c1[mf][j][0], c1[mf][j][1], X.acc[mf][nf][0], b[j].x);
+#pragma unroll
+                for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                    for (int j = 0; j < G::JC; ++j) dmma(c1[mf][j][0], c1[mf][j][1], X.acc[mf][nf][1], b[j].y);
+            }
         }
         // c1[mf][j] = W^T[col mf*8+g][ib (jc+j)*8 + 2t + e]
         double* rw = sm.red + wq * (W * G::LDR);
@@ -149,48 +183,67 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
             for (int j = 0; j < G::JC; ++j)
                 st2(rw + (mf * 8 + g) * G::LDR + (jc + j) * 8 + 2 * t, c1[mf][j][0], c1[mf][j][1]);
     }
-    // T block -> smem (as Tsm[r'*LDT + r] = coefficient of W[r'] in W'[r])
-    for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
-        const int rp = idx / IB, r = idx % IB;
-        double v;
-        if constexpr (TRANS) v = (rp <= r) ? vld<CG>(Ts + r * IB + rp) : 0.0;   // T(r', r), W' = T^T W
-        else                 v = (rp >= r) ? vld<CG>(Ts + rp * IB + r) : 0.0;   // T(r, r'), W' = T W
-        sm.Tsm[rp * G::LDT + r] = v;
-    }
-    __syncthreads();
-    // ---- reduce partials (+ top) -> Wsm (holds W, not yet multiplied by T)
-    for (int idx = threadIdx.x; idx < W * IB; idx += kThreads) {
-        const int col = idx / IB, ib = idx % IB;
-        double s = 0.0;
+    // GEMM2's first V fragments, in flight across the reduction barriers
+    const double* v2 = Vs + rbase + g + (int64_t)t * ldv;
+    double bq[G::NF];
 #pragma unroll
-        for (int w = 0; w < kWarps; ++w) s += sm.red[w * (W * G::LDR) + col * G::LDR + ib];
-        if (top) s += top[(int64_t)col * ldtop + ib];
-        sm.red[col * G::LDR + ib] = s;   // warp-0 slot reused for the reduced W (read-after-sync)
+    for (int nf = 0; nf < G::NF; ++nf) bq[nf] = vld<CG>(v2 + nf * 8);
+#pragma unroll
+    for (int r = 0; r < NT; ++r) {
+        const int idx = tid + r * kThreads;
+        if (idx < IB * IB) sm.Tsm[(idx / IB) * G::LDT + (idx % IB)] = tv[r];
     }
     __syncthreads();
-    // ---- W' = op(T) W;  top -= W';  Wsm = -W'
-    for (int idx = threadIdx.x; idx < W * IB; idx += kThreads) {
-        const int col = idx / IB, r = idx % IB;
-        const double* wc = sm.red + col * G::LDR;
-        double s = 0.0;
+    // ---- (2) reduce the 8 warp partials (+ top) -> red[warp 0 slot]
+#pragma unroll
+    for (int r = 0; r < NR; ++r) {
+        const int idx = tid + r * kThreads;
+        if (idx < W * IB) {
+            const int col = idx / IB, ib = idx % IB;
+            double s = topv[r];
+#pragma unroll
+            for (int w = 0; w < kWarps; ++w) s += sm.red[w * (W * G::LDR) + col * G::LDR + ib];
+            sm.red[col * G::LDR + ib] = s;   // slot 0 entry (col, ib) is read above by this thread only
+        }
+    }
+    __syncthreads();
+    // ---- (3) W' = op(T) W;  top -= W';  Wsm = -W'
+#pragma unroll
+    for (int r = 0; r < NR; ++r) {
+        const int idx = tid + r * kThreads;
+        if (idx < W * IB) {
+            const int col = idx / IB, rr = idx % IB;
+            const double* wc = sm.red + col * G::LDR;
+            double s = 0.0;
 #pragma unroll 8
-        for (int rp = 0; rp < IB; ++rp) s += sm.Tsm[rp * G::LDT + r] * wc[rp];
-        if (top) top[(int64_t)col * ldtop + r] -= s;
-        sm.Wsm[col * G::LDW + r] = -s;
+            for (int rp = 0; rp < IB; ++rp) s += sm.Tsm[rp * G::LDT + rr] * wc[rp];
+            if (top) top[(int64_t)col * ldtop + rr] -= s;
+            sm.Wsm[col * G::LDW + rr] = -s;
+        }
     }
     __syncthreads();
-    // ---- GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row)
+    // ---- (4) GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row), next k-step prefetched
+    double a[G::MF];
+#pragma unroll
+    for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + t];
 #pragma unroll
     for (int kk = 0; kk < IB; kk += 4) {
-        double a[G::MF];
+        double ac[G::MF], bc[G::NF];
 #pragma unroll
-        for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + kk + t];
+        for (int mf = 0; mf < G::MF; ++mf) ac[mf] = a[mf];
+#pragma unroll
+        for (int nf = 0; nf < G::NF; ++nf) bc[nf] = bq[nf];
+        if (kk + 4 < IB) {
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + kk + 4 + t];
+#pragma unroll
+            for (int nf = 0; nf < G::NF; ++nf) bq[nf] = vld<CG>(v2 + (int64_t)(kk + 4) * ldv + nf * 8);
+        }
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
             if (rbase + nf * 8 + 8 <= kmin) continue;
-            const double b = vld<CG>(Vs + (int64_t)(kk + t) * ldv + rbase + nf * 8 + g);
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) dmma(X.acc[mf][nf][0], X.acc[mf][nf][1], a[mf], b);
+            for (int mf = 0; mf < G::MF; ++mf) dmma(X.acc[mf][nf][0], X.acc[mf][nf][1], ac[mf], bc[nf]);
         }
     }
     // Next call writes red before its first __syncthreads; Wsm/Tsm are rewritten only after

@@ -10,9 +10,11 @@
 //   owner(k), panel stream : PANEL(k) = GEQRT(k,k) + TSQRT(k+1..p-1, k)       -> ev_panel[k]
 //   every other owner d    : comm stream receives panel k (peer copy or ncclBroadcast)
 //   owner(k+1), panel str. : lookahead UPDATE(k, column k+1) (waits rest(k-1))   -> ev_look[k]
-//   every owner d, upd str.: UPDATE(k, its columns > k except the lookahead one) -> ev_upd[k]
-// so PANEL(k+1) overlaps the bulk trailing update of step k.  The panel stream has the
-// highest stream priority so freed SMs go to the critical path first.
+//   every owner d, S update streams: UPDATE(k, its columns > k except the lookahead one),
+//                            column lc on stream lc % S                          -> ev_u[u][k]
+// so PANEL(k+1) overlaps the bulk trailing update of step k, and step k+1's updates of one
+// stream start while other streams still finish step k (no wave-quantisation tail per step).
+// The panel stream has the highest stream priority so freed SMs go to the critical path first.
 #include "../../include/tqr.h"
 
 #include <cuda_runtime.h>
@@ -51,9 +53,13 @@ struct Owner {
     unsigned* flags = nullptr;      // p * (nb/ib)
     double* io = nullptr;           // m x (nb*ncols) column-major mirror for host / remote I/O
     cudaStream_t s_panel = nullptr, s_upd = nullptr, s_comm = nullptr;
-    std::vector<cudaEvent_t> ev_panel, ev_recv, ev_upd, ev_look;
-    std::vector<cudaEvent_t> tm0, tm1, tp0, tp1;   // profiling pairs (update rest / panel)
-    std::vector<char> tm_used, tp_used;
+    std::vector<cudaStream_t> s_u;                  // bulk-update streams (column lc -> s_u[lc % S])
+    std::vector<cudaEvent_t> ev_panel, ev_recv, ev_look;
+    std::vector<std::vector<cudaEvent_t>> ev_u;     // ev_u[u][k]: stream u finished its step-k updates
+    std::vector<std::vector<cudaEvent_t>> tm0, tm1; // profiling pairs per (u, k)
+    std::vector<cudaEvent_t> tp0, tp1, tref;        // panel pairs, reference
+    std::vector<std::vector<char>> tm_used;
+    std::vector<char> tp_used;
 };
 
 struct KStat {
@@ -73,6 +79,7 @@ struct tqr_plan_s {
     bool logical = false;
     int rank = 0, world = 1;
     bool lookahead = true, profile = false;
+    int nstreams = 4;               // bulk-update streams per owner (TQR_UPDATE_STREAMS)
     std::vector<Owner> owners;      // in-process: ndev entries; multi-process: 1 (this rank)
     const tqr::NcclApi* nccl = nullptr;
     ncclComm_t comm = nullptr;
@@ -149,8 +156,11 @@ void free_owner(Owner& o) {
     auto F = [](void* p) { if (p) cudaFree(p); };
     F(o.cols_dev); F(o.tiles); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
-    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_upd, &o.ev_look, &o.tm0, &o.tm1, &o.tp0, &o.tp1})
+    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref})
         for (auto e : *v) if (e) cudaEventDestroy(e);
+    for (auto* vv : {&o.ev_u, &o.tm0, &o.tm1})
+        for (auto& v : *vv) for (auto e : v) if (e) cudaEventDestroy(e);
+    for (auto s : o.s_u) if (s) cudaStreamDestroy(s);
     if (o.s_panel) cudaStreamDestroy(o.s_panel);
     if (o.s_upd) cudaStreamDestroy(o.s_upd);
     if (o.s_comm) cudaStreamDestroy(o.s_comm);
@@ -209,6 +219,7 @@ tqr_status sync_all(tqr_plan h) {
         CUDA_TRY(h, cudaStreamSynchronize(o.s_panel));
         CUDA_TRY(h, cudaStreamSynchronize(o.s_upd));
         CUDA_TRY(h, cudaStreamSynchronize(o.s_comm));
+        for (auto su : o.s_u) CUDA_TRY(h, cudaStreamSynchronize(su));
     }
     return TQR_OK;
 }
@@ -302,6 +313,7 @@ tqr_status tqr_destroy(tqr_plan h) {
         if (o.s_panel) cudaStreamSynchronize(o.s_panel);
         if (o.s_upd) cudaStreamSynchronize(o.s_upd);
         if (o.s_comm) cudaStreamSynchronize(o.s_comm);
+        for (auto su : o.s_u) cudaStreamSynchronize(su);
     }
     if (h->comm && h->nccl) h->nccl->CommDestroy(h->comm);
     if (!h->owners.empty()) cudaSetDevice(h->owners[0].dev);
@@ -349,6 +361,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->world = world;
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
+    if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
     h->owner_of.resize(h->q);
     for (int j = 0; j < h->q; ++j) h->owner_of[j] = g[j % g.size()];
 
@@ -371,21 +384,27 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         auto mk = [&](cudaStream_t* s, int prio) { return cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, prio); };
         if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi))
             return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
-        for (auto* v : {&ow.ev_panel, &ow.ev_recv, &ow.ev_upd, &ow.ev_look}) {
-            v->assign(h->q, nullptr);
-            for (auto& e : *v)
-                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                    return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
-        }
-        if (h->profile) {
-            for (auto* v : {&ow.tm0, &ow.tm1, &ow.tp0, &ow.tp1}) {
-                v->assign(h->q, nullptr);
-                for (auto& e : *v)
-                    if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
-            }
-            ow.tm_used.assign(h->q, 0);
+        const int S = h->nstreams;
+        ow.s_u.assign(S, nullptr);
+        for (auto& su : ow.s_u)
+            if (mk(&su, prio_lo)) return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
+        auto mkev = [&](std::vector<cudaEvent_t>& v, int cnt, bool timing) -> bool {
+            v.assign(cnt, nullptr);
+            for (auto& e : v)
+                if ((timing ? cudaEventCreate(&e) : cudaEventCreateWithFlags(&e, cudaEventDisableTiming)) != cudaSuccess)
+                    return false;
+            return true;
+        };
+        bool ok = mkev(ow.ev_panel, h->q, false) && mkev(ow.ev_recv, h->q, false) && mkev(ow.ev_look, h->q, false);
+        ow.ev_u.resize(S);
+        for (int u = 0; u < S && ok; ++u) ok = mkev(ow.ev_u[u], h->q, false);
+        if (ok && h->profile) {
+            ow.tm0.resize(S); ow.tm1.resize(S); ow.tm_used.assign(S, std::vector<char>(h->q, 0));
+            for (int u = 0; u < S && ok; ++u) ok = mkev(ow.tm0[u], h->q, true) && mkev(ow.tm1[u], h->q, true);
+            ok = ok && mkev(ow.tp0, h->q, true) && mkev(ow.tp1, h->q, true) && mkev(ow.tref, 1, true);
             ow.tp_used.assign(h->q, 0);
         }
+        if (!ok) return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
         const size_t nc = ow.cols.size();
         auto alloc = [&](double** ptr, size_t elems) -> bool {
             if (elems == 0) return true;
@@ -497,10 +516,24 @@ tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
 }
 
 // ------------------------------------------------------------------ a2-a7: factor
+namespace {
+// Union length of [t0, t1] intervals (ms) -- device-busy time of one kernel class across streams.
+double union_ms(std::vector<std::pair<double, double>>& iv) {
+    std::sort(iv.begin(), iv.end());
+    double tot = 0.0, cs = -1e300, ce = -1e300;
+    for (auto& x : iv) {
+        if (x.first > ce) { if (ce > cs) tot += ce - cs; cs = x.first; ce = x.second; }
+        else ce = std::max(ce, x.second);
+    }
+    if (ce > cs) tot += ce - cs;
+    return tot;
+}
+}  // namespace
+
 tqr_status tqr_factor_tiles(tqr_plan h) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
-    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
+    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib, S = h->nstreams;
     const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile;
     const unsigned epoch0 = h->epoch;
     h->epoch += (unsigned)q + 1;
@@ -508,15 +541,23 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
     for (auto& o : h->owners) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
         CUDA_TRY(h, cudaStreamSynchronize(o.s_upd));
-        if (h->profile) { std::fill(o.tm_used.begin(), o.tm_used.end(), 0); std::fill(o.tp_used.begin(), o.tp_used.end(), 0); }
+        if (h->profile) {
+            for (auto& v : o.tm_used) std::fill(v.begin(), v.end(), 0);
+            std::fill(o.tp_used.begin(), o.tp_used.end(), 0);
+            CUDA_TRY(h, cudaEventRecord(o.tref[0], o.s_panel));
+        }
     }
+    auto wait_all_u = [&](Owner& D, cudaStream_t st, int kk) -> tqr_status {
+        for (int u = 0; u < S; ++u) CUDA_TRY(h, cudaStreamWaitEvent(st, D.ev_u[u][kk], 0));
+        return TQR_OK;
+    };
     for (int k = 0; k < q; ++k) {
         const int ok = h->owner_of[k];
         Owner* O = h->local(ok);
         // ---- PANEL(k)
         if (O) {
             CUDA_TRY(h, cudaSetDevice(O->dev));
-            if (k > 0 && !h->lookahead) CUDA_TRY(h, cudaStreamWaitEvent(O->s_panel, O->ev_upd[k - 1], 0));
+            if (k > 0 && !h->lookahead) { tqr_status st = wait_all_u(*O, O->s_panel, k - 1); if (st) return st; }
             const int lc = O->lidx[k];
             PanelArgs a;
             a.col = O->tiles + lc * colsz;
@@ -540,7 +581,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             const bool root = (ok == h->rank);
             if (root) CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_panel[k], 0));
             if (!root && k >= 2) {
-                CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_upd[k - 2], 0));
+                tqr_status st = wait_all_u(R, R.s_comm, k - 2);
+                if (st) return st;
                 CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
             }
             double *bt, *bT, *bV;
@@ -550,15 +592,11 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             } else {
                 bt = R.rb_tiles[slot]; bT = R.rb_T[slot]; bV = R.rb_V[slot];
             }
-            const bool need = root || bt != nullptr;
-            double dummy_needed = 0; (void)dummy_needed;
-            if (need) {
-                NCCL_TRY(h, h->nccl->GroupStart());
-                NCCL_TRY(h, h->nccl->Broadcast(bt + k * tile, bt + k * tile, (size_t)(p - k) * tile, ncclFloat64, ok, h->comm, R.s_comm));
-                NCCL_TRY(h, h->nccl->Broadcast(bT + k * tsz, bT + k * tsz, (size_t)(p - k) * tsz, ncclFloat64, ok, h->comm, R.s_comm));
-                NCCL_TRY(h, h->nccl->Broadcast(bV, bV, (size_t)tile, ncclFloat64, ok, h->comm, R.s_comm));
-                NCCL_TRY(h, h->nccl->GroupEnd());
-            }
+            NCCL_TRY(h, h->nccl->GroupStart());
+            NCCL_TRY(h, h->nccl->Broadcast(bt + k * tile, bt + k * tile, (size_t)(p - k) * tile, ncclFloat64, ok, h->comm, R.s_comm));
+            NCCL_TRY(h, h->nccl->Broadcast(bT + k * tsz, bT + k * tsz, (size_t)(p - k) * tsz, ncclFloat64, ok, h->comm, R.s_comm));
+            NCCL_TRY(h, h->nccl->Broadcast(bV, bV, (size_t)tile, ncclFloat64, ok, h->comm, R.s_comm));
+            NCCL_TRY(h, h->nccl->GroupEnd());
             CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
         } else {
             for (auto& D : h->owners) {
@@ -570,7 +608,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 const int slot = k & 1;
                 CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_panel[k], 0));
                 if (k >= 2) {
-                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_upd[k - 2], 0));
+                    tqr_status st = wait_all_u(D, D.s_comm, k - 2);
+                    if (st) return st;
                     CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_look[k - 2], 0));
                 }
                 const int lc = O->lidx[k];
@@ -596,36 +635,44 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 u.V = D.rb_tiles[slot]; u.T = D.rb_T[slot]; u.Vexp = D.rb_V[slot];
             }
             u.X = D.tiles; u.col_stride = colsz; u.tile_stride = tile; u.ld = nb;
-            u.k = k; u.p = p; u.do_unmqr = 1;
+            u.k = k; u.p = p; u.do_unmqr = 1; u.gstride = 1;
             cudaEvent_t ready = mine ? D.ev_panel[k] : D.ev_recv[k];
-            // local columns j > k form a suffix of D.cols
+            // local columns j > k form a suffix [first, ncols) of D.cols
             int first = (int)(std::upper_bound(D.cols.begin(), D.cols.end(), k) - D.cols.begin());
-            int ncols = (int)D.cols.size() - first;
-            const bool la = h->lookahead && ncols > 0 && D.cols[first] == k + 1;
+            const int nloc = (int)D.cols.size();
+            const bool la = h->lookahead && first < nloc && D.cols[first] == k + 1;
             if (la) {
+                // lookahead: column k+1 first, on the high-priority panel stream
                 CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, ready, 0));
-                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_upd[k - 1], 0));
+                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_u[first % S][k - 1], 0));
                 u.group0 = first;
                 CUDA_TRY(h, tqr::launch_update(nb, ib, w_look(h), u, nb / w_look(h), true, D.s_panel));
                 h->launches++;
                 first += 1;
-                ncols -= 1;
             }
             CUDA_TRY(h, cudaEventRecord(D.ev_look[k], D.s_panel));
-            CUDA_TRY(h, cudaStreamWaitEvent(D.s_upd, ready, 0));
-            if (ncols > 0) {
-                u.group0 = first;
-                if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[k], D.s_upd));
-                CUDA_TRY(h, tqr::launch_update(nb, ib, w_bulk(h), u, ncols * (nb / w_bulk(h)), true, D.s_upd));
-                h->launches++;
-                if (h->profile) {
-                    CUDA_TRY(h, cudaEventRecord(D.tm1[k], D.s_upd));
-                    D.tm_used[k] = 1;
-                    h->stats[0].flops += flops_update(h, k, ncols);
-                    h->stats[0].count += 1;
+            // bulk: columns lc in [first, nloc) with lc % S == u on stream u (stream order chains
+            // column lc's step k-1 -> k updates; steps overlap across streams)
+            for (int uu = 0; uu < S; ++uu) {
+                int g0 = first + ((uu - first % S) + S) % S;
+                const int ng = (g0 < nloc) ? (nloc - g0 + S - 1) / S : 0;
+                cudaStream_t su = D.s_u[uu];
+                if (ng > 0) {
+                    CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
+                    u.group0 = g0;
+                    u.gstride = S;
+                    if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[uu][k], su));
+                    CUDA_TRY(h, tqr::launch_update(nb, ib, w_bulk(h), u, ng * (nb / w_bulk(h)), true, su));
+                    h->launches++;
+                    if (h->profile) {
+                        CUDA_TRY(h, cudaEventRecord(D.tm1[uu][k], su));
+                        D.tm_used[uu][k] = 1;
+                        h->stats[0].flops += flops_update(h, k, ng);
+                        h->stats[0].count += 1;
+                    }
                 }
+                CUDA_TRY(h, cudaEventRecord(D.ev_u[uu][k], su));
             }
-            CUDA_TRY(h, cudaEventRecord(D.ev_upd[k], D.s_upd));
         }
     }
     tqr_status st = sync_all(h);
@@ -633,14 +680,25 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
     if (h->profile) {
         for (auto& o : h->owners) {
             CUDA_TRY(h, cudaSetDevice(o.dev));
+            std::vector<std::pair<double, double>> iv, ip;
             for (int k = 0; k < q; ++k) {
-                float ms = 0.f;
-                if (o.tm_used[k]) { CUDA_TRY(h, cudaEventElapsedTime(&ms, o.tm0[k], o.tm1[k])); h->stats[0].ms += ms; }
+                float a = 0.f, b = 0.f;
+                for (int uu = 0; uu < S; ++uu)
+                    if (o.tm_used[uu][k]) {
+                        CUDA_TRY(h, cudaEventElapsedTime(&a, o.tref[0], o.tm0[uu][k]));
+                        CUDA_TRY(h, cudaEventElapsedTime(&b, o.tref[0], o.tm1[uu][k]));
+                        iv.push_back({a, b});
+                    }
                 if (o.tp_used[k]) {
-                    CUDA_TRY(h, cudaEventElapsedTime(&ms, o.tp0[k], o.tp1[k]));
-                    h->stats[1].ms += ms; h->stats[1].count += 1; h->stats[1].flops += flops_panel(h, k);
+                    CUDA_TRY(h, cudaEventElapsedTime(&a, o.tref[0], o.tp0[k]));
+                    CUDA_TRY(h, cudaEventElapsedTime(&b, o.tref[0], o.tp1[k]));
+                    ip.push_back({a, b});
+                    h->stats[1].count += 1;
+                    h->stats[1].flops += flops_panel(h, k);
                 }
             }
+            h->stats[0].ms += union_ms(iv);
+            h->stats[1].ms += union_ms(ip);
         }
     }
     h->factored = true;
@@ -706,7 +764,7 @@ static tqr_status apply_device(tqr_plan h, char trans, double* Bw, int64_t ldw, 
         UpdateArgs u;
         u.V = O->tiles + lc * colsz; u.T = O->T + lc * (int64_t)p * tsz; u.Vexp = O->Vexp + lc * tile;
         u.X = Bw; u.col_stride = (int64_t)nb * ldw; u.tile_stride = nb; u.ld = ldw;
-        u.group0 = 0; u.k = k; u.p = p; u.do_unmqr = 1;
+        u.group0 = 0; u.gstride = 1; u.k = k; u.p = p; u.do_unmqr = 1;
         CUDA_TRY(h, tqr::launch_update(nb, ib, 32, u, (int)nslices, fwd, s));
         h->launches++;
     }

@@ -29,6 +29,7 @@ struct UpdateArgs {
     int64_t tile_stride;
     int64_t ld;
     int group0;          // first group index
+    int gstride;         // group index step between consecutive groups of this launch
     int k, p;
     int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
 };
