@@ -48,6 +48,20 @@ __device__ __forceinline__ double ld_cg(const double* p) {
     return v;
 }
 
+// cp.async (LDGSTS) 16-byte copies global -> shared, grouped per thread.  CG variant caches in
+// L2 only (data published by sibling CTAs of the same grid is never stale in L1).
+template <bool CG>
+__device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+    if constexpr (CG)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
+    else
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
 // Inter-CTA flags (panel kernel wavefront).  Publisher: data stores, __threadfence, then a
 // release store.  Consumer: acquire spin by one thread, fence, then __syncthreads.
 __device__ __forceinline__ void flag_release(unsigned* f, unsigned v) {

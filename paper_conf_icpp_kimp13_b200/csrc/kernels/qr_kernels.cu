@@ -38,13 +38,14 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         X.load_cg(Ai + (int64_t)b * IB * NB, NB);
         for (int bp = 0; bp < b; ++bp) {
             flag_wait_geq(a.flags + (int64_t)i * NBLK + bp, a.epoch);
+            const double* Vb = ge ? a.Vexp + (int64_t)bp * IB * NB : Ai + (int64_t)bp * IB * NB;
+            stage_block<NB, IB, IB, true>(sm, Vb, NB);
             if (ge)
-                apply_block<NB, IB, IB, true, true>(X, sm, a.Vexp + (int64_t)bp * IB * NB, NB,
-                                                    Ti + (int64_t)bp * IB * IB, nullptr, 0, bp * IB);
+                apply_block<NB, IB, IB, true, true>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB, nullptr, 0, bp * IB,
+                                                    nullptr);
             else
-                apply_block<NB, IB, IB, true, true>(X, sm, Ai + (int64_t)bp * IB * NB, NB,
-                                                    Ti + (int64_t)bp * IB * IB,
-                                                    Akk + (int64_t)b * IB * NB + bp * IB, NB, 0);
+                apply_block<NB, IB, IB, true, true>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB,
+                                                    Akk + (int64_t)b * IB * NB + bp * IB, NB, 0, nullptr);
         }
         if (ge) {
             factor_block<NB, IB, true>(X, sm, b * IB);
@@ -104,45 +105,34 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     const int64_t vtile = (int64_t)NB * NB;
     Slice<NB, W, IB> X;
 
-    auto unmqr = [&]() {
-        X.load(Xk, a.ld);
-        const double* Tk = a.T + (int64_t)a.k * IB * NB;
-        if (TRANS) {
-            for (int s = 0; s < NBLK; ++s)
-                apply_block<NB, W, IB, TRANS, false>(X, sm, a.Vexp + (int64_t)s * IB * NB, NB,
-                                                     Tk + (int64_t)s * IB * IB, nullptr, 0, s * IB);
-        } else {
-            for (int s = NBLK - 1; s >= 0; --s)
-                apply_block<NB, W, IB, TRANS, false>(X, sm, a.Vexp + (int64_t)s * IB * NB, NB,
-                                                     Tk + (int64_t)s * IB * IB, nullptr, 0, s * IB);
-        }
-        X.store(Xk, a.ld);
-        __syncthreads();
+    // Reflector blocks in application order; block q of the sequence is staged (cp.async) while
+    // block q-1's GEMM2 runs.  Forward: UNMQR blocks 0..NBLK-1, then for i = k+1..p-1 blocks
+    // 0..NBLK-1 of V_i.  Backward: i = p-1..k+1 blocks NBLK-1..0, then UNMQR blocks NBLK-1..0.
+    const int ntiles = a.p - a.k - 1 + (a.do_unmqr ? 1 : 0);
+    auto tile_of = [&](int q) -> int {            // q-th tile of the sequence; -1 = UNMQR (row tile k)
+        if (TRANS) return a.do_unmqr ? (q == 0 ? -1 : a.k + q) : a.k + 1 + q;
+        return (q < a.p - a.k - 1) ? a.p - 1 - q : -1;
     };
-    auto tsmqr = [&](int i) {
-        double* Xi = Xg + (int64_t)i * a.tile_stride;
-        const double* Vi = a.V + (int64_t)i * vtile;
-        const double* Ti = a.T + (int64_t)i * IB * NB;
+    auto vblock = [&](int ti, int s) -> const double* {
+        return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * vtile) + (int64_t)s * IB * NB;
+    };
+    auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
+    if (ntiles > 0) stage_block<NB, W, IB, false>(sm, vblock(tile_of(0), blk(0)), NB);
+    for (int q = 0; q < ntiles; ++q) {
+        const int ti = tile_of(q);
+        double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
+        const double* Tt = a.T + (int64_t)(ti < 0 ? a.k : ti) * IB * NB;
         X.load(Xi, a.ld);
-        if (TRANS) {
-            for (int s = 0; s < NBLK; ++s)
-                apply_block<NB, W, IB, TRANS, false>(X, sm, Vi + (int64_t)s * IB * NB, NB,
-                                                     Ti + (int64_t)s * IB * IB, Xk + s * IB, a.ld, 0);
-        } else {
-            for (int s = NBLK - 1; s >= 0; --s)
-                apply_block<NB, W, IB, TRANS, false>(X, sm, Vi + (int64_t)s * IB * NB, NB,
-                                                     Ti + (int64_t)s * IB * IB, Xk + s * IB, a.ld, 0);
+        for (int si = 0; si < NBLK; ++si) {
+            const int s = blk(si);
+            const double* nxt = nullptr;
+            if (si + 1 < NBLK) nxt = vblock(ti, blk(si + 1));
+            else if (q + 1 < ntiles) nxt = vblock(tile_of(q + 1), blk(0));
+            apply_block<NB, W, IB, TRANS, false>(X, sm, vblock(ti, s), NB, Tt + (int64_t)s * IB * IB,
+                                                 ti < 0 ? nullptr : Xk + s * IB, a.ld, ti < 0 ? s * IB : 0, nxt);
         }
         X.store(Xi, a.ld);
-    };
-
-    if (TRANS) {
-        if (a.do_unmqr) unmqr();
-        for (int i = a.k + 1; i < a.p; ++i) tsmqr(i);
-    } else {
-        for (int i = a.p - 1; i > a.k; --i) tsmqr(i);
-        __syncthreads();
-        if (a.do_unmqr) unmqr();
+        __syncthreads();   // row tile k (the TS "top") is re-read by other threads
     }
 }
 

@@ -31,21 +31,34 @@ struct Geom {
     static constexpr int NF = RW / 8;        // 8-row fragments per warp
     static constexpr int MF = W / 8;         // 8-column fragments
     static constexpr int JF = IB / 8;        // 8-wide ib fragments
-    static constexpr int JC = (JF < 2) ? JF : 2;  // ib fragments per GEMM1 pass (register budget)
-    static constexpr int LDR = IB + 8;       // red[w][col][ib]   (== 8 mod 16: conflict-free v2 stores)
-    static constexpr int LDW = IB + 4;       // Wsm[col][ib]      (== 4 mod 16: conflict-free A-frag loads)
-    static constexpr int LDT = IB;           // Tsm[r'][r]
-    static_assert(NB % 64 == 0 && W % 8 == 0 && IB % 8 == 0 && NB % IB == 0, "tile geometry");
-    static_assert(IB % (8 * JC) == 0, "ib chunking");
+    static constexpr int HC = IB / 2;        // ib columns per V staging half
+    static constexpr int JC = JF / 2;        // ib fragments per GEMM1 pass (one pass per half)
+    static constexpr int LDR = IB + 8;       // red[slot][col][ib]  (== 8 mod 16: conflict-free v2 stores)
+    static constexpr int LDW = IB + 4;       // Wsm[col][ib]        (== 4 mod 16: conflict-free A-frag loads)
+    static constexpr int LDT = IB;           // Tsm[i][c] (factor output)
+    static constexpr int LDT2 = IB + 2;      // Traw[c][r'] (cp.async target, 16-byte aligned columns)
+    static constexpr int SWZ = (RW >= 16) ? 4 : 0;   // V staging: 16-byte chunk index ^= SWZ*(col&1)
+    static constexpr int VSTN = kWarps * 2 * HC * RW;
+    static constexpr int REDN = 4 * W * LDR;
+    static constexpr int GRAMN = kWarps * IB * LDR;      // factor_block Gram partials (Vst+red+pad)
+    static constexpr int PADN = (GRAMN > VSTN + REDN) ? GRAMN - VSTN - REDN : 2;
+    static_assert(NB % 64 == 0 && W % 8 == 0 && IB % 16 == 0 && NB % IB == 0, "tile geometry");
 };
 
 // Shared-memory workspace of one CTA (apply + factor).  Placed in dynamic smem.
+//   Vst  : per-warp staging of the warp's RW rows of the current V block, two ib-halves
+//          (cp.async, swizzled so GEMM1's 16-byte and GEMM2's 8-byte fragment reads are
+//          conflict-free / 2-way); half A of block s+1 streams in while GEMM2 uses half B of s.
+//   red  : 4 slots of W x IB GEMM1 partials (8 warps reduced in two stages).
 template <int NB, int W, int IB>
 struct Smem {
     using G = Geom<NB, W, IB>;
-    double red[kWarps * W * G::LDR];   // per-warp GEMM partials
-    double Wsm[W * G::LDW];            // -T^T W  (A operand of GEMM2), element (ib, col) at col*LDW + ib
-    double Tsm[IB * G::LDT];           // T block, element used as Tsm[r'*LDT + r]
+    double Vst[kWarps][2][G::HC][G::RW];
+    double red[G::REDN];
+    double gram_pad[G::PADN];          // Vst..gram_pad is the contiguous Gram scratch of factor_block
+    double Wsm[W * G::LDW];            // -op(T) W  (A operand of GEMM2), element (ib, col) at col*LDW + ib
+    double Traw[IB * G::LDT2];         // T block s, element (r', r) at r*LDT2 + r'
+    double Tsm[IB * G::LDT];           // factor_block output T(i, c) at i*LDT + c
     double Rsm[IB * IB];               // TSQRT diagonal R block (row c, col j) at c*IB + j
     double tau[IB];
     double wvec[IB];
@@ -92,38 +105,68 @@ struct Slice {
     }
 };
 
-// V loads: the panel kernel reads V published by sibling CTAs of the same grid -> L2 (.cg);
-// the update kernel reads V that is immutable during the launch -> read-only path (.nc).
-template <bool CG>
-__device__ __forceinline__ double2 vld2(const double* p) {
-    if constexpr (CG) return ld2_cg(p); else return __ldg(reinterpret_cast<const double2*>(p));
+// Element (r, c) of one warp's staging half: chunk-swizzled column-major.
+template <int NB, int W, int IB>
+__device__ __forceinline__ int vst_off(int r, int c) {
+    using G = Geom<NB, W, IB>;
+    return c * G::RW + 2 * ((r >> 1) ^ (G::SWZ * (c & 1))) + (r & 1);
 }
-template <bool CG>
-__device__ __forceinline__ double vld(const double* p) {
-    if constexpr (CG) return ld_cg(p); else return __ldg(p);
+
+// Issue (cp.async + commit) half h of this warp's rows of the V block Vs (NB x IB, ld ldv).
+template <int NB, int W, int IB, bool CG>
+__device__ __forceinline__ void stage_half(Smem<NB, W, IB>& sm, const double* Vs, int64_t ldv, int h) {
+    using G = Geom<NB, W, IB>;
+    constexpr int CPC = G::RW / 2;                 // 16-byte chunks per column
+    constexpr int NCH = G::HC * CPC;               // chunks per half
+    const int lane = lane_id(), wq = warp_id();
+    const double* src = Vs + (int64_t)(h * G::HC) * ldv + wq * G::RW;
+    double* dst = &sm.Vst[wq][h][0][0];
+#pragma unroll
+    for (int q = 0; q < (NCH + 31) / 32; ++q) {
+        const int id = lane + 32 * q;
+        if (NCH % 32 == 0 || id < NCH) {
+            const int c = id / CPC, r2 = id % CPC;
+            cp_async16<CG>(dst + c * G::RW + 2 * (r2 ^ (G::SWZ * (c & 1))), src + (int64_t)c * ldv + 2 * r2);
+        }
+    }
+    cp_async_commit();
+}
+template <int NB, int W, int IB, bool CG>
+__device__ __forceinline__ void stage_block(Smem<NB, W, IB>& sm, const double* Vs, int64_t ldv) {
+    stage_half<NB, W, IB, CG>(sm, Vs, ldv, 0);
+    stage_half<NB, W, IB, CG>(sm, Vs, ldv, 1);
 }
 
 // ---------------------------------------------------------------- apply one ib block
 // X (registers, NB x W) <- H_s X where H_s = I - V_s T_s^T V_s^T (TRANS) or I - V_s T_s V_s^T.
 //   Vs   : column s*IB of V (NB x IB, ld = ldv); rows < kmin are zero (their DMMAs skipped).
-//   Ts   : T block s (IB x IB column-major, ld = IB) = T_tile + s*IB*IB.
+//          Its two halves must already be staged (stage_block, or `next` of the previous call).
+//   Ts   : T block s (IB x IB column-major, ld = IB) = T_tile + s*IB*IB (zeros below diagonal).
 //   top  : if non-null, the X1 rows (IB x W, element (r, c) at top[c*ldtop + r]).
-// Latency hiding (8 warps/SM only, 254 registers): every global operand is loaded one step
-// ahead of its use -- GEMM1's V fragments one row-fragment ahead, GEMM2's first fragments and
-// the top rows / T block before the reduction barriers, GEMM2's next k-step during the current.
+//   next : V block of the following call (same ldv) -- staged here behind GEMM2 -- or null.
+// Barriers: 4 __syncthreads (2-stage reduction, reduced W, T phase).
 template <int NB, int W, int IB, bool TRANS, bool CG>
 __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>& sm,
                                             const double* __restrict__ Vs, int64_t ldv,
                                             const double* __restrict__ Ts,
-                                            double* top, int64_t ldtop, int kmin) {
+                                            double* top, int64_t ldtop, int kmin,
+                                            const double* next) {
     using G = Geom<NB, W, IB>;
     constexpr int NR = (W * IB + kThreads - 1) / kThreads;     // reduce outputs per thread
-    constexpr int NT = (IB * IB + kThreads - 1) / kThreads;    // T entries per thread
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW;
     const int tid = threadIdx.x;
+    (void)Vs;
 
-    // ---- (0) early loads: top rows and T block (consumed after the first barrier)
+    // ---- (0) T block -> Traw (cp.async group), top rows -> registers
+    {
+        constexpr int TCH = IB * IB / 2;   // 16-byte chunks
+        for (int id = tid; id < TCH; id += kThreads) {
+            const int c = id / (IB / 2), r2 = id % (IB / 2);
+            cp_async16<CG>(&sm.Traw[c * G::LDT2 + 2 * r2], Ts + c * IB + 2 * r2);
+        }
+        cp_async_commit();
+    }
     double topv[NR];
 #pragma unroll
     for (int r = 0; r < NR; ++r) {
@@ -131,123 +174,130 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
         topv[r] = 0.0;
         if (top && idx < W * IB) topv[r] = top[(int64_t)(idx / IB) * ldtop + (idx % IB)];
     }
-    double tv[NT];
-#pragma unroll
-    for (int r = 0; r < NT; ++r) {
-        const int idx = tid + r * kThreads;
-        tv[r] = 0.0;
-        if (idx < IB * IB) {
-            const int rp = idx / IB, rr = idx % IB;
-            if constexpr (TRANS) { if (rp <= rr) tv[r] = vld<CG>(Ts + rr * IB + rp); }   // T(r', r): W' = T^T W
-            else                 { if (rp >= rr) tv[r] = vld<CG>(Ts + rp * IB + rr); }   // T(r, r'): W' = T W
-        }
-    }
 
-    // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib)
+    // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib), one pass per half
+    double c1[2][G::MF][G::JC][2];
 #pragma unroll
-    for (int jc = 0; jc < G::JF; jc += G::JC) {
-        double c1[G::MF][G::JC][2];
+    for (int h = 0; h < 2; ++h) {
+        if (h == 0) cp_async_wait<2>(); else cp_async_wait<1>();   // pending: [A, B, T] -> A done / B done
+        __syncwarp();
+        const double* vh = &sm.Vst[wq][h][0][0];
 #pragma unroll
         for (int mf = 0; mf < G::MF; ++mf)
 #pragma unroll
-            for (int j = 0; j < G::JC; ++j) c1[mf][j][0] = c1[mf][j][1] = 0.0;
-        const double* vb = Vs + (int64_t)(jc * 8 + g) * ldv + rbase + 2 * t;
-        double2 bn[G::JC];
-#pragma unroll
-        for (int j = 0; j < G::JC; ++j) bn[j] = vld2<CG>(vb + (int64_t)j * 8 * ldv);
+            for (int j = 0; j < G::JC; ++j) c1[h][mf][j][0] = c1[h][mf][j][1] = 0.0;
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
+            if (rbase + nf * 8 + 8 <= kmin) continue;        // V rows all zero (warp-uniform)
             double2 b[G::JC];
 #pragma unroll
-            for (int j = 0; j < G::JC; ++j) b[j] = bn[j];
-            if (nf + 1 < G::NF) {
-#pragma unroll
-                for (int j = 0; j < G::JC; ++j) bn[j] = vld2<CG>(vb + (int64_t)j * 8 * ldv + (nf + 1) * 8);
-            }
-            if (rbase + nf * 8 + 8 > kmin) {                 // rows < kmin of V are zero
-#pragma unroll
-                for (int mf = 0; mf < G::MF; ++mf)
-#pragma unroll
-                    for (int j = 0; j < G::JC; ++j) dmma(c1[mf][j][0], c1[mf][j][1], X.acc[mf][nf][0], b[j].x);
-#pragma unroll
-                for (int mf = 0; mf < G::MF; ++mf)
-#pragma unroll
-                    for (int j = 0; j < G::JC; ++j) dmma(c1[mf][j][0], c1[mf][j][1], X.acc[mf][nf][1], b[j].y);
-            }
-        }
-        // c1[mf][j] = W^T[col mf*8+g][ib (jc+j)*8 + 2t + e]
-        double* rw = sm.red + wq * (W * G::LDR);
-#pragma unroll
-        for (int mf = 0; mf < G::MF; ++mf)
-#pragma unroll
             for (int j = 0; j < G::JC; ++j)
-                st2(rw + (mf * 8 + g) * G::LDR + (jc + j) * 8 + 2 * t, c1[mf][j][0], c1[mf][j][1]);
+                b[j] = *reinterpret_cast<const double2*>(vh + vst_off<NB, W, IB>(nf * 8 + 2 * t, j * 8 + g));
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                for (int j = 0; j < G::JC; ++j) dmma(c1[h][mf][j][0], c1[h][mf][j][1], X.acc[mf][nf][0], b[j].x);
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                for (int j = 0; j < G::JC; ++j) dmma(c1[h][mf][j][0], c1[h][mf][j][1], X.acc[mf][nf][1], b[j].y);
+        }
     }
-    // GEMM2's first V fragments, in flight across the reduction barriers
-    const double* v2 = Vs + rbase + g + (int64_t)t * ldv;
-    double bq[G::NF];
+    // c1[h][mf][j] = W^T[col mf*8+g][ib h*HC + j*8 + 2t + e]
+    // ---- (2) two-stage reduction of the 8 warp partials: warps 4..7 store, warps 0..3 add
+    auto frag_ptr = [&](int slot, int h, int mf, int j) {
+        return sm.red + slot * (W * G::LDR) + (mf * 8 + g) * G::LDR + h * G::HC + j * 8 + 2 * t;
+    };
+    if (wq >= 4) {
 #pragma unroll
-    for (int nf = 0; nf < G::NF; ++nf) bq[nf] = vld<CG>(v2 + nf * 8);
+        for (int h = 0; h < 2; ++h)
 #pragma unroll
-    for (int r = 0; r < NT; ++r) {
-        const int idx = tid + r * kThreads;
-        if (idx < IB * IB) sm.Tsm[(idx / IB) * G::LDT + (idx % IB)] = tv[r];
+            for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                for (int j = 0; j < G::JC; ++j) st2(frag_ptr(wq - 4, h, mf, j), c1[h][mf][j][0], c1[h][mf][j][1]);
     }
     __syncthreads();
-    // ---- (2) reduce the 8 warp partials (+ top) -> red[warp 0 slot]
+    if (wq < 4) {
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                for (int j = 0; j < G::JC; ++j) {
+                    double* pp = frag_ptr(wq, h, mf, j);
+                    const double2 o = *reinterpret_cast<const double2*>(pp);
+                    st2(pp, o.x + c1[h][mf][j][0], o.y + c1[h][mf][j][1]);
+                }
+    }
+    __syncthreads();
 #pragma unroll
     for (int r = 0; r < NR; ++r) {
         const int idx = tid + r * kThreads;
         if (idx < W * IB) {
             const int col = idx / IB, ib = idx % IB;
-            double s = topv[r];
+            const double* rp = sm.red + col * G::LDR + ib;
+            const double s = topv[r] + ((rp[0] + rp[W * G::LDR]) + (rp[2 * W * G::LDR] + rp[3 * W * G::LDR]));
+            sm.red[col * G::LDR + ib] = s;   // slot-0 entry (col, ib) is read above by this thread only
+        }
+    }
+    cp_async_wait<0>();                      // T block (and both V halves) landed for this thread
+    __syncthreads();
+    // ---- (3) W'^T = W^T op(T)^T on DMMA (W x IB output, 8x8 fragments spread over the warps):
+    //      C[m = col][n = r] = sum_k W^T[col][k] B[k][n],  B = T (TRANS: W' = T^T W) or T^T.
+    //      Wsm = -W'.  T has explicit zeros off its triangle.
+    {
+        constexpr int NFRAG = G::MF * G::JF;
+        for (int f = wq; f < NFRAG; f += kWarps) {
+            const int mf = f / G::JF, jf = f % G::JF;
+            double c0 = 0.0, c1v = 0.0;
+            const double* wa = sm.red + (mf * 8 + g) * G::LDR + t;
 #pragma unroll
-            for (int w = 0; w < kWarps; ++w) s += sm.red[w * (W * G::LDR) + col * G::LDR + ib];
-            sm.red[col * G::LDR + ib] = s;   // slot 0 entry (col, ib) is read above by this thread only
+            for (int kk = 0; kk < IB; kk += 4) {
+                const double av = wa[kk];
+                double bv;
+                if constexpr (TRANS) bv = sm.Traw[(jf * 8 + g) * G::LDT2 + kk + t];   // T(kk+t, r)
+                else                 bv = sm.Traw[(kk + t) * G::LDT2 + jf * 8 + g];   // T(r, kk+t)
+                dmma(c0, c1v, av, bv);
+            }
+            st2(&sm.Wsm[(mf * 8 + g) * G::LDW + jf * 8 + 2 * t], -c0, -c1v);
         }
     }
     __syncthreads();
-    // ---- (3) W' = op(T) W;  top -= W';  Wsm = -W'
+    // top -= W'  (top + Wsm, same per-thread mapping as the reduction; original top in topv)
+    if (top) {
 #pragma unroll
-    for (int r = 0; r < NR; ++r) {
-        const int idx = tid + r * kThreads;
-        if (idx < W * IB) {
-            const int col = idx / IB, rr = idx % IB;
-            const double* wc = sm.red + col * G::LDR;
-            double s = 0.0;
-#pragma unroll 8
-            for (int rp = 0; rp < IB; ++rp) s += sm.Tsm[rp * G::LDT + rr] * wc[rp];
-            if (top) top[(int64_t)col * ldtop + rr] -= s;
-            sm.Wsm[col * G::LDW + rr] = -s;
+        for (int r = 0; r < NR; ++r) {
+            const int idx = tid + r * kThreads;
+            if (idx < W * IB) {
+                const int col = idx / IB, rr = idx % IB;
+                top[(int64_t)col * ldtop + rr] = topv[r] + sm.Wsm[col * G::LDW + rr];
+            }
         }
     }
-    __syncthreads();
-    // ---- (4) GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row), next k-step prefetched
-    double a[G::MF];
+    // ---- (4) GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row); stage `next` behind each half
 #pragma unroll
-    for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + t];
+    for (int h = 0; h < 2; ++h) {
+        const double* vh = &sm.Vst[wq][h][0][0];
 #pragma unroll
-    for (int kk = 0; kk < IB; kk += 4) {
-        double ac[G::MF], bc[G::NF];
+        for (int kk = 0; kk < G::HC; kk += 4) {
+            double a[G::MF];
 #pragma unroll
-        for (int mf = 0; mf < G::MF; ++mf) ac[mf] = a[mf];
+            for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + h * G::HC + kk + t];
 #pragma unroll
-        for (int nf = 0; nf < G::NF; ++nf) bc[nf] = bq[nf];
-        if (kk + 4 < IB) {
+            for (int nf = 0; nf < G::NF; ++nf) {
+                if (rbase + nf * 8 + 8 <= kmin) continue;
+                const double b = vh[vst_off<NB, W, IB>(nf * 8 + g, kk + t)];
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + kk + 4 + t];
-#pragma unroll
-            for (int nf = 0; nf < G::NF; ++nf) bq[nf] = vld<CG>(v2 + (int64_t)(kk + 4) * ldv + nf * 8);
+                for (int mf = 0; mf < G::MF; ++mf) dmma(X.acc[mf][nf][0], X.acc[mf][nf][1], a[mf], b);
+            }
         }
-#pragma unroll
-        for (int nf = 0; nf < G::NF; ++nf) {
-            if (rbase + nf * 8 + 8 <= kmin) continue;
-#pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) dmma(X.acc[mf][nf][0], X.acc[mf][nf][1], ac[mf], bc[nf]);
+        if (next) {
+            __syncwarp();
+            stage_half<NB, W, IB, CG>(sm, next, ldv, h);
         }
     }
-    // Next call writes red before its first __syncthreads; Wsm/Tsm are rewritten only after
-    // that barrier, which every warp reaches after finishing this GEMM2.
+    // The next call's first barrier is preceded only by warp-private Vst reads and red stores
+    // into slots that every warp finished reading before this call's last barrier.
 }
 
 // ---------------------------------------------------------------- factor ib columns
@@ -391,7 +441,10 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                     for (int j = 0; j < G::MF; ++j) dmma(gacc[i][j][0], gacc[i][j][1], v[i], v[j]);
             }
         // gacc[i][j] = G[c' = i*8+g][c = j*8 + 2t + e]
-        double* rw = sm.red + wq * (IB * G::LDR);
+        // 8 warp partials in the (idle) V staging + reduction area (contiguous members)
+        static_assert(G::GRAMN <= G::VSTN + G::REDN + G::PADN, "Gram scratch");
+        double* scratch = &sm.Vst[0][0][0][0];
+        double* rw = scratch + wq * (IB * G::LDR);
 #pragma unroll
         for (int i = 0; i < G::MF; ++i)
 #pragma unroll
@@ -402,7 +455,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             const int cp = idx / IB, c = idx % IB;
             double s = 0.0;
 #pragma unroll
-            for (int w = 0; w < kWarps; ++w) s += sm.red[w * (IB * G::LDR) + cp * G::LDR + c];
+            for (int w = 0; w < kWarps; ++w) s += scratch[w * (IB * G::LDR) + cp * G::LDR + c];
             sm.Wsm[cp * G::LDW + c] = s;   // Gram(c', c)
         }
         __syncthreads();
