@@ -43,9 +43,9 @@ def _stale(target, deps):
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def _compile(src):
-    obj = os.path.join(OBJ, os.path.basename(src) + ".o")
-    cmd = [NVCC] + ARCH + COMMON + ["-c", src, "-o", obj]
+def _compile(src, defines=(), tag=""):
+    obj = os.path.join(OBJ, os.path.basename(src) + tag + ".o")
+    cmd = [NVCC] + ARCH + COMMON + ["-D" + d for d in defines] + ["-c", src, "-o", obj]
     if src.endswith(".cpp"):
         cmd = [os.environ.get("CXX", "g++"), "-O3", "-std=c++17", "-g", "-fPIC", "-Wall",
                "-I" + os.path.join(ROOT, "include"), "-I" + CSRC, "-I/usr/local/cuda/include", "-c", src, "-o", obj]
@@ -66,6 +66,16 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if verbose:
         print("built", LIB)
     return LIB
+
+
+def build_variant(name: str, defines) -> str:
+    """Probe-only variant library (e.g. phase-timing instrumentation), never loaded by the product."""
+    os.makedirs(OBJ, exist_ok=True)
+    with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
+        objs = list(ex.map(lambda s: _compile(s, defines, "." + name), SOURCES))
+    out = os.path.join(OBJ, "libtqr_%s.so" % name)
+    subprocess.check_call([NVCC] + ARCH + ["-shared", "-cudart", "static", "-o", out] + objs + ["-ldl", "-lpthread"])
+    return out
 
 
 if __name__ == "__main__":

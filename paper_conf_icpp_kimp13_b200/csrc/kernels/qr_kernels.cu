@@ -23,7 +23,7 @@ namespace tqr {
 template <int NB, int IB>
 __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    auto& sm = *reinterpret_cast<Smem<NB, IB, IB>*>(smem_raw);
+    auto& sm = *reinterpret_cast<Smem<NB, IB, IB, true>*>(smem_raw);
     constexpr int NBLK = NB / IB;
     const int b = blockIdx.x;
     const int64_t tile = (int64_t)NB * NB;
@@ -39,13 +39,13 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         for (int bp = 0; bp < b; ++bp) {
             flag_wait_geq(a.flags + (int64_t)i * NBLK + bp, a.epoch);
             const double* Vb = ge ? a.Vexp + (int64_t)bp * IB * NB : Ai + (int64_t)bp * IB * NB;
-            stage_block<NB, IB, IB, true>(sm, Vb, NB);
+            stage_first<NB, IB, IB, true, true>(sm, Vb, NB);
             if (ge)
-                apply_block<NB, IB, IB, true, true>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB, nullptr, 0, bp * IB,
-                                                    nullptr);
+                apply_block<NB, IB, IB, true, true, true, true>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB, nullptr,
+                                                                0, bp * IB, nullptr);
             else
-                apply_block<NB, IB, IB, true, true>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB,
-                                                    Akk + (int64_t)b * IB * NB + bp * IB, NB, 0, nullptr);
+                apply_block<NB, IB, IB, true, true, true, false>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB,
+                                                                 Akk + (int64_t)b * IB * NB + bp * IB, NB, 0, nullptr);
         }
         if (ge) {
             factor_block<NB, IB, true>(X, sm, b * IB);
@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
 template <int NB, int W, int IB, bool TRANS>
 __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    auto& sm = *reinterpret_cast<Smem<NB, W, IB>*>(smem_raw);
+    auto& sm = *reinterpret_cast<Smem<NB, W, IB, false>*>(smem_raw);
     constexpr int SPG = NB / W;     // slices per column group
     constexpr int NBLK = NB / IB;
     const int grp = blockIdx.x / SPG;
@@ -117,7 +117,7 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
         return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * vtile) + (int64_t)s * IB * NB;
     };
     auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
-    if (ntiles > 0) stage_block<NB, W, IB, false>(sm, vblock(tile_of(0), blk(0)), NB);
+    if (ntiles > 0) stage_first<NB, W, IB, false, false>(sm, vblock(tile_of(0), blk(0)), NB);
     for (int q = 0; q < ntiles; ++q) {
         const int ti = tile_of(q);
         double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
@@ -128,8 +128,12 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
             const double* nxt = nullptr;
             if (si + 1 < NBLK) nxt = vblock(ti, blk(si + 1));
             else if (q + 1 < ntiles) nxt = vblock(tile_of(q + 1), blk(0));
-            apply_block<NB, W, IB, TRANS, false>(X, sm, vblock(ti, s), NB, Tt + (int64_t)s * IB * IB,
-                                                 ti < 0 ? nullptr : Xk + s * IB, a.ld, ti < 0 ? s * IB : 0, nxt);
+            if (ti < 0)
+                apply_block<NB, W, IB, false, TRANS, false, true>(X, sm, vblock(ti, s), NB, Tt + (int64_t)s * IB * IB,
+                                                                  nullptr, a.ld, s * IB, nxt);
+            else
+                apply_block<NB, W, IB, false, TRANS, false, false>(X, sm, vblock(ti, s), NB, Tt + (int64_t)s * IB * IB,
+                                                                   Xk + s * IB, a.ld, 0, nxt);
         }
         X.store(Xi, a.ld);
         __syncthreads();   // row tile k (the TS "top") is re-read by other threads
@@ -215,7 +219,7 @@ __global__ void zero_diag_check_kernel(const double* __restrict__ R, int64_t ldr
 // ============================================================================ launchers
 template <int NB, int IB>
 static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s) {
-    const size_t smem = sizeof(Smem<NB, IB, IB>);
+    const size_t smem = sizeof(Smem<NB, IB, IB, true>);
     auto kern = panel_kernel<NB, IB>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -225,7 +229,7 @@ static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s) {
 
 template <int NB, int W, int IB>
 static cudaError_t launch_update_t(const UpdateArgs& a, int nslices, bool trans, cudaStream_t s) {
-    const size_t smem = sizeof(Smem<NB, W, IB>);
+    const size_t smem = sizeof(Smem<NB, W, IB, false>);
     const int grid = nslices;
     if (grid <= 0) return cudaSuccess;
     if (trans) {
@@ -321,7 +325,7 @@ cudaError_t launch_zero_diag_check(const double* R, int64_t ldr, int64_t n, int6
 }
 
 size_t panel_smem_bytes(int nb, int ib) {
-#define TQR_PS(NB_, IB_) if (nb == NB_ && ib == IB_) return sizeof(Smem<NB_, IB_, IB_>);
+#define TQR_PS(NB_, IB_) if (nb == NB_ && ib == IB_) return sizeof(Smem<NB_, IB_, IB_, true>);
     TQR_PS(64, 16) TQR_PS(64, 32) TQR_PS(128, 16) TQR_PS(128, 32)
     TQR_PS(256, 16) TQR_PS(256, 32) TQR_PS(512, 16) TQR_PS(512, 32)
 #undef TQR_PS
@@ -330,9 +334,9 @@ size_t panel_smem_bytes(int nb, int ib) {
 
 size_t update_smem_bytes(int nb, int ib, int w) {
 #define TQR_US(NB_, IB_) if (nb == NB_ && ib == IB_) { \
-        if (w == 8) return sizeof(Smem<NB_, 8, IB_>); \
-        if (w == 16) return sizeof(Smem<NB_, 16, IB_>); \
-        if (w == 32) return sizeof(Smem<NB_, 32, IB_>); }
+        if (w == 8) return sizeof(Smem<NB_, 8, IB_, false>); \
+        if (w == 16) return sizeof(Smem<NB_, 16, IB_, false>); \
+        if (w == 32) return sizeof(Smem<NB_, 32, IB_, false>); }
     TQR_US(64, 16) TQR_US(64, 32) TQR_US(128, 16) TQR_US(128, 32)
     TQR_US(256, 16) TQR_US(256, 32) TQR_US(512, 16) TQR_US(512, 32)
 #undef TQR_US
@@ -340,3 +344,14 @@ size_t update_smem_bytes(int nb, int ib, int w) {
 }
 
 }  // namespace tqr
+
+#ifdef TQR_PHASE_PROF
+extern "C" int tqr_probe_phases(unsigned long long* out, int reset) {
+    cudaMemcpyFromSymbol(out, tqr::g_phase, sizeof(unsigned long long) * 16);
+    if (reset) {
+        unsigned long long z[16] = {0};
+        cudaMemcpyToSymbol(tqr::g_phase, z, sizeof(z));
+    }
+    return (int)cudaGetLastError();
+}
+#endif

@@ -22,6 +22,17 @@
 
 namespace tqr {
 
+#ifdef TQR_PHASE_PROF
+// Probe-only instrumentation (tools/probes): per-phase clock64 totals of warp 0 of every CTA.
+__device__ unsigned long long g_phase[16];
+#define TQR_PH(i) do { if ((threadIdx.x & 255) == 0) { long long _c = clock64(); \
+    atomicAdd(&g_phase[i], (unsigned long long)(_c - _ph)); _ph = _c; } } while (0)
+#define TQR_PH0() long long _ph = clock64()
+#else
+#define TQR_PH(i) do {} while (0)
+#define TQR_PH0() do {} while (0)
+#endif
+
 constexpr int kThreads = 256;
 constexpr int kWarps = 8;
 
@@ -33,33 +44,38 @@ struct Geom {
     static constexpr int JF = IB / 8;        // 8-wide ib fragments
     static constexpr int HC = IB / 2;        // ib columns per V staging half
     static constexpr int JC = JF / 2;        // ib fragments per GEMM1 pass (one pass per half)
-    static constexpr int LDR = IB + 8;       // red[slot][col][ib]  (== 8 mod 16: conflict-free v2 stores)
-    static constexpr int LDW = IB + 4;       // Wsm[col][ib]        (== 4 mod 16: conflict-free A-frag loads)
+    static constexpr int LDR = IB + 4;       // red[slot][col][ib]
+    static constexpr int LDW = IB + 4;       // Wsm[col][ib]      (== 4 mod 16: conflict-free A-frag loads)
     static constexpr int LDT = IB;           // Tsm[i][c] (factor output)
     static constexpr int LDT2 = IB + 2;      // Traw[c][r'] (cp.async target, 16-byte aligned columns)
     static constexpr int SWZ = (RW >= 16) ? 4 : 0;   // V staging: 16-byte chunk index ^= SWZ*(col&1)
+    static constexpr int CPC = RW / 2;       // 16-byte chunks per staged column
+    static constexpr int NQ = (HC * CPC + 31) / 32;   // chunks per lane per half
     static constexpr int VSTN = kWarps * 2 * HC * RW;
-    static constexpr int REDN = 4 * W * LDR;
-    static constexpr int GRAMN = kWarps * IB * LDR;      // factor_block Gram partials (Vst+red+pad)
-    static constexpr int PADN = (GRAMN > VSTN + REDN) ? GRAMN - VSTN - REDN : 2;
+    static constexpr int GRAMN = kWarps * IB * LDR;  // factor_block Gram partials (Vst + red + pad)
     static_assert(NB % 64 == 0 && W % 8 == 0 && IB % 16 == 0 && NB % IB == 0, "tile geometry");
 };
 
-// Shared-memory workspace of one CTA (apply + factor).  Placed in dynamic smem.
+// Shared-memory workspace of one CTA.  FACT = panel kernel (factor_block members, 4-slot
+// two-stage reduction); !FACT = update kernel (8-slot single-stage reduction).
 //   Vst  : per-warp staging of the warp's RW rows of the current V block, two ib-halves
 //          (cp.async, swizzled so GEMM1's 16-byte and GEMM2's 8-byte fragment reads are
-//          conflict-free / 2-way); half A of block s+1 streams in while GEMM2 uses half B of s.
-//   red  : 4 slots of W x IB GEMM1 partials (8 warps reduced in two stages).
-template <int NB, int W, int IB>
+//          conflict-free / 2-way).  Half B of block s is issued inside GEMM1's half-A loop and
+//          half A of block s+1 inside GEMM2's half-B loop, so the copies overlap DMMA issue.
+//   red  : NSLOT slots of W x IB GEMM1 partials.
+template <int NB, int W, int IB, bool FACT>
 struct Smem {
     using G = Geom<NB, W, IB>;
+    static constexpr int NSLOT = FACT ? 4 : 8;
+    static constexpr int REDN = NSLOT * W * G::LDR;
+    static constexpr int PADN = (FACT && G::GRAMN > G::VSTN + REDN) ? G::GRAMN - G::VSTN - REDN : 2;
     double Vst[kWarps][2][G::HC][G::RW];
-    double red[G::REDN];
-    double gram_pad[G::PADN];          // Vst..gram_pad is the contiguous Gram scratch of factor_block
+    double red[REDN];
+    double gram_pad[PADN];             // Vst..gram_pad is the contiguous Gram scratch of factor_block
     double Wsm[W * G::LDW];            // -op(T) W  (A operand of GEMM2), element (ib, col) at col*LDW + ib
     double Traw[IB * G::LDT2];         // T block s, element (r', r) at r*LDT2 + r'
-    double Tsm[IB * G::LDT];           // factor_block output T(i, c) at i*LDT + c
-    double Rsm[IB * IB];               // TSQRT diagonal R block (row c, col j) at c*IB + j
+    double Tsm[FACT ? IB * G::LDT : 2];   // factor_block output T(i, c) at i*LDT + c
+    double Rsm[FACT ? IB * IB : 2];       // TSQRT diagonal R block (row c, col j) at c*IB + j
     double tau[IB];
     double wvec[IB];
     double red1[kWarps];
@@ -112,61 +128,57 @@ __device__ __forceinline__ int vst_off(int r, int c) {
     return c * G::RW + 2 * ((r >> 1) ^ (G::SWZ * (c & 1))) + (r & 1);
 }
 
-// Issue (cp.async + commit) half h of this warp's rows of the V block Vs (NB x IB, ld ldv).
-template <int NB, int W, int IB, bool CG>
-__device__ __forceinline__ void stage_half(Smem<NB, W, IB>& sm, const double* Vs, int64_t ldv, int h) {
+// Issue (no commit) this lane's chunks q in [q0, q1) of half h of this warp's rows of Vs.
+template <int NB, int W, int IB, bool FACT, bool CG>
+__device__ __forceinline__ void stage_part(Smem<NB, W, IB, FACT>& sm, const double* Vs, int64_t ldv, int h,
+                                           int q0, int q1) {
     using G = Geom<NB, W, IB>;
-    constexpr int CPC = G::RW / 2;                 // 16-byte chunks per column
-    constexpr int NCH = G::HC * CPC;               // chunks per half
+    constexpr int NCH = G::HC * G::CPC;
     const int lane = lane_id(), wq = warp_id();
     const double* src = Vs + (int64_t)(h * G::HC) * ldv + wq * G::RW;
     double* dst = &sm.Vst[wq][h][0][0];
 #pragma unroll
-    for (int q = 0; q < (NCH + 31) / 32; ++q) {
+    for (int q = 0; q < G::NQ; ++q) {
+        if (q < q0 || q >= q1) continue;
         const int id = lane + 32 * q;
         if (NCH % 32 == 0 || id < NCH) {
-            const int c = id / CPC, r2 = id % CPC;
+            const int c = id / G::CPC, r2 = id % G::CPC;
             cp_async16<CG>(dst + c * G::RW + 2 * (r2 ^ (G::SWZ * (c & 1))), src + (int64_t)c * ldv + 2 * r2);
         }
     }
-    cp_async_commit();
 }
-template <int NB, int W, int IB, bool CG>
-__device__ __forceinline__ void stage_block(Smem<NB, W, IB>& sm, const double* Vs, int64_t ldv) {
-    stage_half<NB, W, IB, CG>(sm, Vs, ldv, 0);
-    stage_half<NB, W, IB, CG>(sm, Vs, ldv, 1);
+// Prologue of a block sequence: half A of the first block (one cp.async group).
+template <int NB, int W, int IB, bool FACT, bool CG>
+__device__ __forceinline__ void stage_first(Smem<NB, W, IB, FACT>& sm, const double* Vs, int64_t ldv) {
+    stage_part<NB, W, IB, FACT, CG>(sm, Vs, ldv, 0, 0, Geom<NB, W, IB>::NQ);
+    cp_async_commit();
 }
 
 // ---------------------------------------------------------------- apply one ib block
 // X (registers, NB x W) <- H_s X where H_s = I - V_s T_s^T V_s^T (TRANS) or I - V_s T_s V_s^T.
 //   Vs   : column s*IB of V (NB x IB, ld = ldv); rows < kmin are zero (their DMMAs skipped).
-//          Its two halves must already be staged (stage_block, or `next` of the previous call).
+//          Half A must be in flight (stage_first, or `next` of the previous call).
 //   Ts   : T block s (IB x IB column-major, ld = IB) = T_tile + s*IB*IB (zeros below diagonal).
 //   top  : if non-null, the X1 rows (IB x W, element (r, c) at top[c*ldtop + r]).
-//   next : V block of the following call (same ldv) -- staged here behind GEMM2 -- or null.
-// Barriers: 4 __syncthreads (2-stage reduction, reduced W, T phase).
-template <int NB, int W, int IB, bool TRANS, bool CG>
-__device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>& sm,
+//   next : V block of the following call (same ldv) -- its half A is staged here -- or null.
+//   KM   : kmin may be > 0 (UNMQR / GEQRT blocks); false compiles the TS path branch-free.
+template <int NB, int W, int IB, bool FACT, bool TRANS, bool CG, bool KM>
+__device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB, FACT>& sm,
                                             const double* __restrict__ Vs, int64_t ldv,
                                             const double* __restrict__ Ts,
                                             double* top, int64_t ldtop, int kmin,
                                             const double* next) {
     using G = Geom<NB, W, IB>;
+    using SM = Smem<NB, W, IB, FACT>;
     constexpr int NR = (W * IB + kThreads - 1) / kThreads;     // reduce outputs per thread
+    constexpr int NQ = G::NQ;
+    constexpr int QH = (NQ + 1) / 2;                           // chunks per lane per issue step
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW;
     const int tid = threadIdx.x;
-    (void)Vs;
+    TQR_PH0();
 
-    // ---- (0) T block -> Traw (cp.async group), top rows -> registers
-    {
-        constexpr int TCH = IB * IB / 2;   // 16-byte chunks
-        for (int id = tid; id < TCH; id += kThreads) {
-            const int c = id / (IB / 2), r2 = id % (IB / 2);
-            cp_async16<CG>(&sm.Traw[c * G::LDT2 + 2 * r2], Ts + c * IB + 2 * r2);
-        }
-        cp_async_commit();
-    }
+    // ---- (0) top rows -> registers (consumed after the reduction barrier)
     double topv[NR];
 #pragma unroll
     for (int r = 0; r < NR; ++r) {
@@ -174,13 +186,15 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
         topv[r] = 0.0;
         if (top && idx < W * IB) topv[r] = top[(int64_t)(idx / IB) * ldtop + (idx % IB)];
     }
+    cp_async_wait<0>();                       // half A of this block
+    __syncwarp();
+    TQR_PH(0);
 
     // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib), one pass per half
     double c1[2][G::MF][G::JC][2];
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-        if (h == 0) cp_async_wait<2>(); else cp_async_wait<1>();   // pending: [A, B, T] -> A done / B done
-        __syncwarp();
+        if (h == 1) { cp_async_wait<0>(); __syncwarp(); }   // half B + T block
         const double* vh = &sm.Vst[wq][h][0][0];
 #pragma unroll
         for (int mf = 0; mf < G::MF; ++mf)
@@ -188,7 +202,21 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
             for (int j = 0; j < G::JC; ++j) c1[h][mf][j][0] = c1[h][mf][j][1] = 0.0;
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
-            if (rbase + nf * 8 + 8 <= kmin) continue;        // V rows all zero (warp-uniform)
+            if (h == 0 && nf == 0) {
+                // overlap: T block and the first part of half B behind these DMMAs
+                constexpr int TCH = IB * IB / 2;   // 16-byte chunks of the T block
+                for (int id = tid; id < TCH; id += kThreads) {
+                    const int c = id / (IB / 2), r2 = id % (IB / 2);
+                    cp_async16<CG>(&sm.Traw[c * G::LDT2 + 2 * r2], Ts + c * IB + 2 * r2);
+                }
+                stage_part<NB, W, IB, FACT, CG>(sm, Vs, ldv, 1, 0, G::NF > 1 ? QH : NQ);
+                if (G::NF == 1) cp_async_commit();
+            }
+            if (h == 0 && nf == 1) {
+                stage_part<NB, W, IB, FACT, CG>(sm, Vs, ldv, 1, QH, NQ);
+                cp_async_commit();
+            }
+            if (KM && rbase + nf * 8 + 8 <= kmin) continue;  // V rows all zero (warp-uniform)
             double2 b[G::JC];
 #pragma unroll
             for (int j = 0; j < G::JC; ++j)
@@ -202,46 +230,66 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
 #pragma unroll
                 for (int j = 0; j < G::JC; ++j) dmma(c1[h][mf][j][0], c1[h][mf][j][1], X.acc[mf][nf][1], b[j].y);
         }
+        TQR_PH(1 + h);
     }
     // c1[h][mf][j] = W^T[col mf*8+g][ib h*HC + j*8 + 2t + e]
-    // ---- (2) two-stage reduction of the 8 warp partials: warps 4..7 store, warps 0..3 add
+    // ---- (2) cross-warp reduction of the 8 partials (+ top) into slot 0
     auto frag_ptr = [&](int slot, int h, int mf, int j) {
         return sm.red + slot * (W * G::LDR) + (mf * 8 + g) * G::LDR + h * G::HC + j * 8 + 2 * t;
     };
-    if (wq >= 4) {
+    if constexpr (SM::NSLOT == 8) {
 #pragma unroll
         for (int h = 0; h < 2; ++h)
 #pragma unroll
             for (int mf = 0; mf < G::MF; ++mf)
 #pragma unroll
-                for (int j = 0; j < G::JC; ++j) st2(frag_ptr(wq - 4, h, mf, j), c1[h][mf][j][0], c1[h][mf][j][1]);
+                for (int j = 0; j < G::JC; ++j) st2(frag_ptr(wq, h, mf, j), c1[h][mf][j][0], c1[h][mf][j][1]);
+        __syncthreads();
+        TQR_PH(3);
+    } else {   // 4 slots: warps 4..7 store, warps 0..3 add
+        if (wq >= 4) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+                for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                    for (int j = 0; j < G::JC; ++j) st2(frag_ptr(wq - 4, h, mf, j), c1[h][mf][j][0], c1[h][mf][j][1]);
+        }
+        __syncthreads();
+        TQR_PH(3);
+        if (wq < 4) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+                for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                    for (int j = 0; j < G::JC; ++j) {
+                        double* pp = frag_ptr(wq, h, mf, j);
+                        const double2 o = *reinterpret_cast<const double2*>(pp);
+                        st2(pp, o.x + c1[h][mf][j][0], o.y + c1[h][mf][j][1]);
+                    }
+        }
+        __syncthreads();
     }
-    __syncthreads();
-    if (wq < 4) {
-#pragma unroll
-        for (int h = 0; h < 2; ++h)
-#pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf)
-#pragma unroll
-                for (int j = 0; j < G::JC; ++j) {
-                    double* pp = frag_ptr(wq, h, mf, j);
-                    const double2 o = *reinterpret_cast<const double2*>(pp);
-                    st2(pp, o.x + c1[h][mf][j][0], o.y + c1[h][mf][j][1]);
-                }
-    }
-    __syncthreads();
+    TQR_PH(4);
 #pragma unroll
     for (int r = 0; r < NR; ++r) {
         const int idx = tid + r * kThreads;
         if (idx < W * IB) {
             const int col = idx / IB, ib = idx % IB;
             const double* rp = sm.red + col * G::LDR + ib;
-            const double s = topv[r] + ((rp[0] + rp[W * G::LDR]) + (rp[2 * W * G::LDR] + rp[3 * W * G::LDR]));
-            sm.red[col * G::LDR + ib] = s;   // slot-0 entry (col, ib) is read above by this thread only
+            double s = 0.0;
+            if constexpr (SM::NSLOT == 8) {
+                s = ((rp[0] + rp[W * G::LDR]) + (rp[2 * W * G::LDR] + rp[3 * W * G::LDR])) +
+                    ((rp[4 * W * G::LDR] + rp[5 * W * G::LDR]) + (rp[6 * W * G::LDR] + rp[7 * W * G::LDR]));
+            } else {
+                s = (rp[0] + rp[W * G::LDR]) + (rp[2 * W * G::LDR] + rp[3 * W * G::LDR]);
+            }
+            sm.red[col * G::LDR + ib] = topv[r] + s;   // slot-0 entry (col, ib) is read above by this thread only
         }
     }
-    cp_async_wait<0>();                      // T block (and both V halves) landed for this thread
     __syncthreads();
+    TQR_PH(5);
     // ---- (3) W'^T = W^T op(T)^T on DMMA (W x IB output, 8x8 fragments spread over the warps):
     //      C[m = col][n = r] = sum_k W^T[col][k] B[k][n],  B = T (TRANS: W' = T^T W) or T^T.
     //      Wsm = -W'.  T has explicit zeros off its triangle.
@@ -263,7 +311,8 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
         }
     }
     __syncthreads();
-    // top -= W'  (top + Wsm, same per-thread mapping as the reduction; original top in topv)
+    TQR_PH(6);
+    // top -= W'  (original top in topv, same per-thread mapping as the reduction)
     if (top) {
 #pragma unroll
         for (int r = 0; r < NR; ++r) {
@@ -274,30 +323,40 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
             }
         }
     }
-    // ---- (4) GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row); stage `next` behind each half
+    TQR_PH(7);
+    // ---- (4) GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row); half A of `next` staged
+    //      inside the half-B loop (half A of this block is no longer read there)
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
+        if (h == 1) __syncwarp();
         const double* vh = &sm.Vst[wq][h][0][0];
 #pragma unroll
         for (int kk = 0; kk < G::HC; kk += 4) {
+            if (h == 1 && next != nullptr) {
+                if (kk == 0) {
+                    stage_part<NB, W, IB, FACT, CG>(sm, next, ldv, 0, 0, G::HC > 4 ? QH : NQ);
+                    if (G::HC <= 4) cp_async_commit();
+                } else if (kk == 4) {
+                    stage_part<NB, W, IB, FACT, CG>(sm, next, ldv, 0, QH, NQ);
+                    cp_async_commit();
+                }
+            }
             double a[G::MF];
 #pragma unroll
             for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + h * G::HC + kk + t];
 #pragma unroll
             for (int nf = 0; nf < G::NF; ++nf) {
-                if (rbase + nf * 8 + 8 <= kmin) continue;
+                if (KM && rbase + nf * 8 + 8 <= kmin) continue;
                 const double b = vh[vst_off<NB, W, IB>(nf * 8 + g, kk + t)];
 #pragma unroll
                 for (int mf = 0; mf < G::MF; ++mf) dmma(X.acc[mf][nf][0], X.acc[mf][nf][1], a[mf], b);
             }
         }
-        if (next) {
-            __syncwarp();
-            stage_half<NB, W, IB, CG>(sm, next, ldv, h);
-        }
+        TQR_PH(8 + h);
     }
-    // The next call's first barrier is preceded only by warp-private Vst reads and red stores
-    // into slots that every warp finished reading before this call's last barrier.
+    // Exit: at most one cp.async group (half A of `next`) pending.  The next call's first
+    // barrier is preceded only by warp-private Vst traffic and red stores into slots that every
+    // warp finished reading before this call's last barrier.
 }
 
 // ---------------------------------------------------------------- factor ib columns
@@ -307,7 +366,7 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB>
 // all NB rows of X are the dense V2 part.  On exit: X = reflectors, sm.tau, sm.Tsm holds the
 // IB x IB T factor as Tsm[i*LDT + c] = T(i, c) (upper triangle, zeros below).
 template <int NB, int IB, bool GE>
-__device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, IB>& sm, int dbase) {
+__device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, IB, true>& sm, int dbase) {
     using G = Geom<NB, IB, IB>;
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW + 2 * t;   // row of acc[.][nf][e] = rbase + nf*8 + e
@@ -442,7 +501,8 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             }
         // gacc[i][j] = G[c' = i*8+g][c = j*8 + 2t + e]
         // 8 warp partials in the (idle) V staging + reduction area (contiguous members)
-        static_assert(G::GRAMN <= G::VSTN + G::REDN + G::PADN, "Gram scratch");
+        using SM = Smem<NB, IB, IB, true>;
+        static_assert(G::GRAMN <= G::VSTN + SM::REDN + SM::PADN, "Gram scratch");
         double* scratch = &sm.Vst[0][0][0][0];
         double* rw = scratch + wq * (IB * G::LDR);
 #pragma unroll
