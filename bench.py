@@ -12,7 +12,7 @@ e2e    : the same through tqr_factor-equivalent calls on PINNED HOST buffers (H2
 N > 1  : launched by torchrun; one process per GPU, column tiles partitioned by the guide
          array {0..N-1} (Eq. 12), panels broadcast with NCCL.  Strong scaling (same matrix).
 --impl reference : the CPU oracle (Algorithm 1, oracle/) timed on this host's cores on a
-         bounded sample of the same workload (first 512 columns of the config's matrix).
+         bounded sample of the same workload (first 2048 columns of the config's matrix).
 """
 from __future__ import annotations
 
@@ -38,6 +38,7 @@ CONFIGS = {
 }
 DEFAULT_CONFIG = "C5"
 L2_BYTES = 126 * 2 ** 20
+SAMPLE_COLS = int(os.environ.get("TQR_ORACLE_SAMPLE_COLS", "2048"))
 
 
 def flops(m, n):
@@ -52,6 +53,15 @@ def fp64_peak_tflops():
         return float(d["dmma_tflops"]), d.get("source", "profiles/fp64_peak.json")
     except Exception:
         return 37.2, "nominal 148 SM x 64 FMA/clk x 2 x 1.965 GHz"
+
+
+def load_profile_summary(cfg):
+    """ncu summary of the dominant kernel for this config (profiles/ncu_update_<cfg>.json)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_update_%s.json" % cfg)) as f:
+            return json.load(f)
+    except Exception:
+        return {}
 
 
 class ClockSampler:
@@ -106,13 +116,14 @@ class ClockSampler:
 
 
 def oracle_sample(cfg_name, nthreads=0):
-    """Bounded CPU-oracle sample of the config: Algorithm 1 on the first min(n, 512) columns
-    of the config's own matrix (same generator, same rows).  Returns (GFLOP/s, seconds, desc)."""
+    """Bounded CPU-oracle sample of the config: Algorithm 1 on the first min(n, 2048) columns
+    of the config's own matrix (same generator, same rows; ~10 s of host work for C5).
+    Returns (GFLOP/s, seconds, desc)."""
     import numpy as np
     import oracle
     import synthetic
     m, n, nb, ib, seed = CONFIGS[cfg_name]
-    ns = min(n, 512)
+    ns = min(n, SAMPLE_COLS)
     rows = np.arange(m, dtype=np.uint64)
     A = np.empty((m, ns), order="F")
     for j in range(ns):
@@ -145,7 +156,7 @@ def run_reference(args):
         "ms_per_step": round(1e3 * statistics.median(times), 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
-                   "sample": "first %d columns" % min(n, 512)},
+                   "sample": "first %d columns" % min(n, SAMPLE_COLS)},
         "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
                          "sample": desc},
         "e2e": {"value": round(value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -273,9 +284,7 @@ def main():
                "sample": desc}
 
     if rank == 0:
-        upd_ms = ums / max(ucount, 1)
-        upd_fl = uflops / max(ucount, 1)
-        achieved = (upd_fl / (upd_ms * 1e-3) / 1e12) if ucount else None
+        achieved = (uflops / (ums * 1e-3) / 1e12) if ucount else None
         line = {
             "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak",
             "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
@@ -287,10 +296,13 @@ def main():
                        "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
                        "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (8 * m * n / 2 ** 30)
                        if 8 * m * n > L2_BYTES else "input fits L2 (no flush)"},
-            "roofline": {"bound": "tensor", "kernel": "update_kernel (UNMQR+TSMQR, DMMA.8x8x4)",
+            "roofline": {"bound": "tensor", "kernel": "update_kernel<512,32,32> (UNMQR+TSMQR chain, DMMA.8x8x4)",
                          "achieved": round(achieved, 3) if achieved else None, "peak": peak, "unit": "TFLOP/s",
-                         "frac": round(achieved / peak, 4) if achieved else None, "traffic": None,
-                         "peak_source": peak_src, "launches": ucount, "avg_ms": round(upd_ms, 3),
+                         "frac": round(achieved / peak, 4) if achieved else None,
+                         "traffic": prof.get("dram_bytes_per_launch"),
+                         "traffic_note": prof.get("note"),
+                         "peak_source": peak_src, "launches_per_step": ucount // K,
+                         "busy_ms_per_step": round(ums / K, 3),
                          "share_of_step": round(ums / K / ms, 3) if ucount else None},
             "panel": {"launches": pcount, "avg_ms": round(pms / max(pcount, 1), 3),
                       "tflops": round(pflops / max(pms, 1e-9) / 1e9, 3) if pcount else None},
