@@ -284,7 +284,11 @@ def main():
                "sample": desc}
 
     if rank == 0:
+        # achieved = algorithmic flops of all bulk-update launches / their device-busy time
+        # (union of the launches' CUDA-event intervals on the 4 update streams; the launches of
+        # one step overlap, so a per-launch average duration would not be a kernel duration)
         achieved = (uflops / (ums * 1e-3) / 1e12) if ucount else None
+        prof = load_profile_summary(args.config)
         line = {
             "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak",
             "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,

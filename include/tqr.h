@@ -52,8 +52,9 @@ typedef struct {
      * guide-array partition and broadcast ordering on one GPU.  0: owner d uses CUDA
      * device d (single-process) or this process's device (multi-process). */
     int32_t logical_devices;
-    /* Multi-process mode (one process per GPU): world > 1, this process is `rank`; ndev must
-     * equal world.  nccl_id points to the 128-byte ncclUniqueId produced by
+    /* Multi-process (NCCL) mode, one process per GPU: world > 1 (or world <= 1 with a non-NULL
+     * nccl_id: a single-rank communicator), this process is `rank`; ndev must equal
+     * max(world, 1).  nccl_id points to the 128-byte ncclUniqueId produced by
      * tqr_nccl_unique_id() on rank 0 and shared out of band (e.g. torch.distributed). */
     int32_t rank;
     int32_t world;

@@ -94,7 +94,8 @@ struct tqr_plan_s {
     double* rcm = nullptr;
     int64_t* dflag = nullptr;
 
-    bool multiproc() const { return world > 1; }
+    bool nccl_mode = false;         // one process per GPU, panels broadcast with NCCL
+    bool multiproc() const { return nccl_mode; }
     Owner* local(int d) {
         if (multiproc()) return (d == rank) ? &owners[0] : nullptr;
         return &owners[d];
@@ -342,23 +343,26 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     if (dtype != TQR_F64) return fail(nullptr, TQR_ERR_UNSUPPORTED, "FP32 path not in this build");
     tqr_options o{};
     if (opt) o = *opt;
+    // NCCL mode: world > 1, or a single-rank communicator when an nccl_id is given explicitly
+    const bool use_nccl = o.world > 1 || o.nccl_id != nullptr;
     const int world = o.world > 1 ? o.world : 1;
-    if (world > 1 && (o.rank < 0 || o.rank >= world || ndev != world || !o.nccl_id))
+    if (use_nccl && (o.rank < 0 || o.rank >= world || ndev != world || !o.nccl_id))
         return fail(nullptr, TQR_ERR_ARG, "multi-process: need 0 <= rank < world == ndev and nccl_id");
     int ndevices = 0;
     if (cudaGetDeviceCount(&ndevices) != cudaSuccess || ndevices < 1) {
         cudaGetLastError();
         return fail(nullptr, TQR_ERR_CUDA, "no CUDA device");
     }
-    if (world == 1 && !o.logical_devices && ndev > ndevices)
+    if (!use_nccl && !o.logical_devices && ndev > ndevices)
         return fail(nullptr, TQR_ERR_ARG, "ndev %d > %d visible CUDA devices (set logical_devices)", ndev, ndevices);
 
     tqr_plan h = new tqr_plan_s();
     h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)(m / nb); h->q = (int)(n / nb);
     h->dtype = dtype; h->ndev = ndev; h->guide = g;
     h->logical = o.logical_devices != 0;
-    h->rank = world > 1 ? o.rank : 0;
+    h->rank = use_nccl ? o.rank : 0;
     h->world = world;
+    h->nccl_mode = use_nccl;
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
@@ -367,7 +371,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
 
     int cur = 0;
     cudaGetDevice(&cur);
-    const int nown = world > 1 ? 1 : ndev;
+    const int nown = use_nccl ? 1 : ndev;
     h->owners.resize(nown);
     auto bail = [&](tqr_status s) { std::string e = h->err; tqr_destroy(h); g_create_error = e; return s; };
     int prio_lo = 0, prio_hi = 0;
@@ -375,8 +379,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     const int64_t p = h->p, tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb;
     for (int li = 0; li < nown; ++li) {
         Owner& ow = h->owners[li];
-        ow.id = world > 1 ? h->rank : li;
-        ow.dev = (world > 1 || h->logical) ? cur : li;
+        ow.id = use_nccl ? h->rank : li;
+        ow.dev = (use_nccl || h->logical) ? cur : li;
         ow.lidx.assign(h->q, -1);
         for (int j = 0; j < h->q; ++j)
             if (h->owner_of[j] == ow.id) { ow.lidx[j] = (int32_t)ow.cols.size(); ow.cols.push_back(j); }
@@ -421,7 +425,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
                 return bail(fail(h, TQR_ERR_ALLOC, "cols allocation failed"));
         }
         // receive slots are needed when some remote panel k precedes an owned column
-        bool need_rb = world > 1;   // every rank takes part in every ncclBroadcast
+        bool need_rb = use_nccl;    // every rank takes part in every ncclBroadcast
         for (int k = 0; k < h->q && !need_rb; ++k)
             if (h->owner_of[k] != ow.id)
                 for (int j = k + 1; j < h->q; ++j) if (h->owner_of[j] == ow.id) { need_rb = true; break; }
@@ -437,7 +441,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         }
     }
     // peer access between physical owners (single-process, several GPUs)
-    if (world == 1 && !h->logical && ndev > 1) {
+    if (!use_nccl && !h->logical && ndev > 1) {
         for (int a = 0; a < ndev; ++a)
             for (int b = 0; b < ndev; ++b) {
                 if (a == b) continue;
@@ -446,7 +450,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
                 if (can) { cudaSetDevice(a); cudaDeviceEnablePeerAccess(b, 0); cudaGetLastError(); }
             }
     }
-    if (world > 1) {
+    if (use_nccl) {
         const char* why = nullptr;
         h->nccl = tqr::nccl_api(&why);
         if (!h->nccl) return bail(fail(h, TQR_ERR_NCCL, "NCCL unavailable: %s", why));
