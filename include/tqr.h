@@ -17,7 +17,9 @@
  *   - Pointers may be host memory (pageable or pinned) or device memory of the plan's
  *     first device; the library detects which with cudaPointerGetAttributes.  The caller
  *     owns its buffers; the plan never frees or retains them past the call.
- *   - Calls are synchronous: on return every result is in the caller's buffer.
+ *   - Calls are synchronous: each call that touches a caller buffer first waits for all work
+ *     already queued on the buffer's / plan's devices (any stream), and on return every result
+ *     is in the caller's buffer.
  *   - A CUDA or NCCL failure poisons the plan: later calls return TQR_ERR_STATE until
  *     tqr_destroy.  A plan is not thread-safe; distinct plans are independent.
  */

@@ -24,12 +24,16 @@ template <int NB, int IB>
 __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     auto& sm = *reinterpret_cast<Smem<NB, IB, IB, true>*>(smem_raw);
+    using G = Geom<NB, IB, IB>;
     constexpr int NBLK = NB / IB;
     const int b = blockIdx.x;
     const int64_t tile = (int64_t)NB * NB;
     double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
     double* Akk = col + (int64_t)a.k * tile;
     Slice<NB, IB, IB> X;
+    stage_init(sm);
+    unsigned vph = 0;
+    const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
 
     for (int i = a.k; i < a.p; ++i) {
         double* Ai = col + (int64_t)i * tile;
@@ -38,14 +42,16 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         X.load_cg(Ai + (int64_t)b * IB * NB, NB);
         for (int bp = 0; bp < b; ++bp) {
             flag_wait_geq(a.flags + (int64_t)i * NBLK + bp, a.epoch);
-            const double* Vb = ge ? a.Vexp + (int64_t)bp * IB * NB : Ai + (int64_t)bp * IB * NB;
-            stage_first<NB, IB, IB, true, true>(sm, Vb, NB);
+            const double* Vb = (ge ? a.Vexp : a.Vimg + (int64_t)i * tile) + (int64_t)bp * IB * NB;
+            if (lane_id() == 0) fence_proxy_async_global();   // sibling CTA's generic stores -> bulk copy
+            stage_first(sm, Vb);
             if (ge)
-                apply_block<NB, IB, IB, true, true, true, true>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB, nullptr,
-                                                                0, bp * IB, nullptr);
+                apply_block<NB, IB, IB, true, true, true, true>(X, sm, Vb, Ti + (int64_t)bp * IB * IB, nullptr, 0,
+                                                                bp * IB, nullptr, vph);
             else
-                apply_block<NB, IB, IB, true, true, true, false>(X, sm, Vb, NB, Ti + (int64_t)bp * IB * IB,
-                                                                 Akk + (int64_t)b * IB * NB + bp * IB, NB, 0, nullptr);
+                apply_block<NB, IB, IB, true, true, true, false>(X, sm, Vb, Ti + (int64_t)bp * IB * IB,
+                                                                 Akk + (int64_t)b * IB * NB + bp * IB, NB, 0,
+                                                                 nullptr, vph);
         }
         if (ge) {
             factor_block<NB, IB, true>(X, sm, b * IB);
@@ -58,31 +64,37 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
             __syncthreads();
             factor_block<NB, IB, false>(X, sm, b * IB);
         }
-        // publish: reflectors, T block, R block (TSQRT), explicit V (GEQRT)
+        // publish: reflectors (LAPACK layout in the tile), their stage image (TSQRT: V2 of tile i;
+        // GEQRT: explicit unit-lower V of the diagonal tile), the T block, the R block (TSQRT)
         X.store(Ai + (int64_t)b * IB * NB, NB);
         for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
             const int c = idx / IB, r = idx % IB;   // T(r, c) -> column-major block b
             Ti[(int64_t)b * IB * IB + c * IB + r] = sm.Tsm[r * IB + c];
         }
-        if (ge) {
-            const int g = lane_id() >> 2, t = lane_id() & 3, r0 = warp_id() * (NB / 8) + 2 * t;
+        double* img = ge ? a.Vexp : a.Vimg + (int64_t)i * tile;
 #pragma unroll
-            for (int mf = 0; mf < IB / 8; ++mf) {
-                const int dc = b * IB + mf * 8 + g;
+        for (int mf = 0; mf < IB / 8; ++mf) {
+            const int cb = mf * 8 + g;                 // column within the block
+            const int dc = b * IB + cb;                // column within the tile
 #pragma unroll
-                for (int nf = 0; nf < NB / 64; ++nf) {
-                    const int r = r0 + nf * 8;
-                    double v0 = (r > dc) ? X.acc[mf][nf][0] : (r == dc ? 1.0 : 0.0);
-                    double v1 = (r + 1 > dc) ? X.acc[mf][nf][1] : (r + 1 == dc ? 1.0 : 0.0);
-                    st2(a.Vexp + (int64_t)dc * NB + r, v0, v1);
+            for (int nf = 0; nf < G::NF; ++nf) {
+                const int rl = nf * 8 + 2 * t;         // row within this warp's rows
+                const int r = wq * G::RW + rl;
+                double v0 = X.acc[mf][nf][0], v1 = X.acc[mf][nf][1];
+                if (ge) {
+                    v0 = (r > dc) ? v0 : (r == dc ? 1.0 : 0.0);
+                    v1 = (r + 1 > dc) ? v1 : (r + 1 == dc ? 1.0 : 0.0);
                 }
+                st2(img + vimg_off<NB, IB, IB>(b, wq, cb / G::HC, rl, cb % G::HC), v0, v1);
             }
-        } else {
+        }
+        if (!ge) {
             for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
                 const int j = idx / IB, c = idx % IB;
                 if (c <= j) Akk[(int64_t)(b * IB + j) * NB + b * IB + c] = sm.Rsm[c * IB + j];
             }
         }
+        fence_proxy_async_global();
         __threadfence();
         __syncthreads();
         if (threadIdx.x == 0) flag_release(a.flags + (int64_t)i * NBLK + b, a.epoch);
@@ -104,6 +116,8 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     double* Xk = Xg + (int64_t)a.k * a.tile_stride;
     const int64_t vtile = (int64_t)NB * NB;
     Slice<NB, W, IB> X;
+    stage_init(sm);
+    unsigned vph = 0;
 
     // Reflector blocks in application order; block q of the sequence is staged (cp.async) while
     // block q-1's GEMM2 runs.  Forward: UNMQR blocks 0..NBLK-1, then for i = k+1..p-1 blocks
@@ -117,7 +131,7 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
         return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * vtile) + (int64_t)s * IB * NB;
     };
     auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
-    if (ntiles > 0) stage_first<NB, W, IB, false, false>(sm, vblock(tile_of(0), blk(0)), NB);
+    if (ntiles > 0) stage_first(sm, vblock(tile_of(0), blk(0)));
     for (int q = 0; q < ntiles; ++q) {
         const int ti = tile_of(q);
         double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
@@ -129,11 +143,11 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
             if (si + 1 < NBLK) nxt = vblock(ti, blk(si + 1));
             else if (q + 1 < ntiles) nxt = vblock(tile_of(q + 1), blk(0));
             if (ti < 0)
-                apply_block<NB, W, IB, false, TRANS, false, true>(X, sm, vblock(ti, s), NB, Tt + (int64_t)s * IB * IB,
-                                                                  nullptr, a.ld, s * IB, nxt);
+                apply_block<NB, W, IB, false, TRANS, false, true>(X, sm, vblock(ti, s), Tt + (int64_t)s * IB * IB,
+                                                                  nullptr, a.ld, s * IB, nxt, vph);
             else
-                apply_block<NB, W, IB, false, TRANS, false, false>(X, sm, vblock(ti, s), NB, Tt + (int64_t)s * IB * IB,
-                                                                   Xk + s * IB, a.ld, 0, nxt);
+                apply_block<NB, W, IB, false, TRANS, false, false>(X, sm, vblock(ti, s), Tt + (int64_t)s * IB * IB,
+                                                                   Xk + s * IB, a.ld, 0, nxt, vph);
         }
         X.store(Xi, a.ld);
         __syncthreads();   // row tile k (the TS "top") is re-read by other threads

@@ -58,10 +58,12 @@ struct Geom {
 
 // Shared-memory workspace of one CTA.  FACT = panel kernel (factor_block members, 4-slot
 // two-stage reduction); !FACT = update kernel (8-slot single-stage reduction).
-//   Vst  : per-warp staging of the warp's RW rows of the current V block, two ib-halves
-//          (cp.async, swizzled so GEMM1's 16-byte and GEMM2's 8-byte fragment reads are
-//          conflict-free / 2-way).  Half B of block s is issued inside GEMM1's half-A loop and
-//          half A of block s+1 inside GEMM2's half-B loop, so the copies overlap DMMA issue.
+//   Vst  : per-warp staging of the warp's RW rows of the current V block, two ib-halves,
+//          filled by one cp.async.bulk (8 KB at nb=512) per warp and half from the
+//          pre-swizzled "stage image" of V that the panel kernel writes (vimg_off), so the
+//          GEMM1 16-byte / GEMM2 8-byte fragment reads are conflict-free / 2-way with no
+//          per-lane copy instructions.  Half B of block s is issued at the start of block s,
+//          half A of block s+1 as soon as GEMM2 has finished reading half A of block s.
 //   red  : NSLOT slots of W x IB GEMM1 partials.
 template <int NB, int W, int IB, bool FACT>
 struct Smem {
@@ -80,6 +82,7 @@ struct Smem {
     double wvec[IB];
     double red1[kWarps];
     double x0;
+    uint64_t mbar[kWarps][2];          // bulk-copy completion of Vst[w][h] (outside the Gram scratch)
 };
 
 // ---------------------------------------------------------------- register slice I/O
@@ -128,51 +131,59 @@ __device__ __forceinline__ int vst_off(int r, int c) {
     return c * G::RW + 2 * ((r >> 1) ^ (G::SWZ * (c & 1))) + (r & 1);
 }
 
-// Issue (no commit) this lane's chunks q in [q0, q1) of half h of this warp's rows of Vs.
-template <int NB, int W, int IB, bool FACT, bool CG>
-__device__ __forceinline__ void stage_part(Smem<NB, W, IB, FACT>& sm, const double* Vs, int64_t ldv, int h,
-                                           int q0, int q1) {
+// Stage image of a V tile (NB x NB, written by the panel kernel): ib block s, warp rows q, half h
+// is the contiguous HC*RW chunk at s*IB*NB + (q*2 + h)*HC*RW, laid out exactly like Vst[q][h].
+template <int NB, int W, int IB>
+__device__ __forceinline__ int64_t vimg_off(int s, int q, int h, int r, int c) {
     using G = Geom<NB, W, IB>;
-    constexpr int NCH = G::HC * G::CPC;
-    const int lane = lane_id(), wq = warp_id();
-    const double* src = Vs + (int64_t)(h * G::HC) * ldv + wq * G::RW;
-    double* dst = &sm.Vst[wq][h][0][0];
-#pragma unroll
-    for (int q = 0; q < G::NQ; ++q) {
-        if (q < q0 || q >= q1) continue;
-        const int id = lane + 32 * q;
-        if (NCH % 32 == 0 || id < NCH) {
-            const int c = id / G::CPC, r2 = id % G::CPC;
-            cp_async16<CG>(dst + c * G::RW + 2 * (r2 ^ (G::SWZ * (c & 1))), src + (int64_t)c * ldv + 2 * r2);
-        }
+    return (int64_t)s * IB * NB + (q * 2 + h) * (G::HC * G::RW) + vst_off<NB, W, IB>(r, c);
+}
+
+// Per-warp bulk staging of half h of block image `blk` (lane 0 issues; WAR-safe after the
+// warp's own reads of that half: __syncwarp + async-proxy fence).
+template <int NB, int W, int IB, bool FACT>
+__device__ __forceinline__ void stage_bulk(Smem<NB, W, IB, FACT>& sm, const double* blk, int h) {
+    using G = Geom<NB, W, IB>;
+    const int wq = warp_id();
+    __syncwarp();
+    if (lane_id() == 0) {
+        fence_proxy_async_shared();
+        bulk_g2s(&sm.Vst[wq][h][0][0], blk + (wq * 2 + h) * (G::HC * G::RW), G::HC * G::RW * 8, &sm.mbar[wq][h]);
     }
 }
-// Prologue of a block sequence: half A of the first block (one cp.async group).
-template <int NB, int W, int IB, bool FACT, bool CG>
-__device__ __forceinline__ void stage_first(Smem<NB, W, IB, FACT>& sm, const double* Vs, int64_t ldv) {
-    stage_part<NB, W, IB, FACT, CG>(sm, Vs, ldv, 0, 0, Geom<NB, W, IB>::NQ);
-    cp_async_commit();
+template <int NB, int W, int IB, bool FACT>
+__device__ __forceinline__ void stage_init(Smem<NB, W, IB, FACT>& sm) {
+    if (lane_id() == 0) {
+        mbar_init(&sm.mbar[warp_id()][0], 1);
+        mbar_init(&sm.mbar[warp_id()][1], 1);
+        fence_mbar_init();
+    }
+    __syncwarp();
+}
+// Prologue of a block sequence: half A of the first block.
+template <int NB, int W, int IB, bool FACT>
+__device__ __forceinline__ void stage_first(Smem<NB, W, IB, FACT>& sm, const double* blk) {
+    stage_bulk(sm, blk, 0);
 }
 
 // ---------------------------------------------------------------- apply one ib block
 // X (registers, NB x W) <- H_s X where H_s = I - V_s T_s^T V_s^T (TRANS) or I - V_s T_s V_s^T.
-//   Vs   : column s*IB of V (NB x IB, ld = ldv); rows < kmin are zero (their DMMAs skipped).
+//   Vs   : stage image of V block s (vimg_off); rows < kmin are zero (their DMMAs skipped).
 //          Half A must be in flight (stage_first, or `next` of the previous call).
+//   vph  : the warp's mbarrier phase bits (bit h for half h), carried across calls.
 //   Ts   : T block s (IB x IB column-major, ld = IB) = T_tile + s*IB*IB (zeros below diagonal).
 //   top  : if non-null, the X1 rows (IB x W, element (r, c) at top[c*ldtop + r]).
-//   next : V block of the following call (same ldv) -- its half A is staged here -- or null.
+//   next : stage image of the following call's block -- its half A is staged here -- or null.
 //   KM   : kmin may be > 0 (UNMQR / GEQRT blocks); false compiles the TS path branch-free.
 template <int NB, int W, int IB, bool FACT, bool TRANS, bool CG, bool KM>
 __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB, FACT>& sm,
-                                            const double* __restrict__ Vs, int64_t ldv,
+                                            const double* __restrict__ Vs,
                                             const double* __restrict__ Ts,
                                             double* top, int64_t ldtop, int kmin,
-                                            const double* next) {
+                                            const double* next, unsigned& vph) {
     using G = Geom<NB, W, IB>;
     using SM = Smem<NB, W, IB, FACT>;
     constexpr int NR = (W * IB + kThreads - 1) / kThreads;     // reduce outputs per thread
-    constexpr int NQ = G::NQ;
-    constexpr int QH = (NQ + 1) / 2;                           // chunks per lane per issue step
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW;
     const int tid = threadIdx.x;
@@ -186,15 +197,23 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
         topv[r] = 0.0;
         if (top && idx < W * IB) topv[r] = top[(int64_t)(idx / IB) * ldtop + (idx % IB)];
     }
-    cp_async_wait<0>();                       // half A of this block
-    __syncwarp();
+    stage_bulk(sm, Vs, 1);                    // half B of this block (its buffer was read last call)
+    {   // T block -> Traw (LDGSTS group; waited before the reduction barrier)
+        constexpr int TCH = IB * IB / 2;
+        for (int id = tid; id < TCH; id += kThreads) {
+            const int c = id / (IB / 2), r2 = id % (IB / 2);
+            cp_async16<CG>(&sm.Traw[c * G::LDT2 + 2 * r2], Ts + c * IB + 2 * r2);
+        }
+        cp_async_commit();
+    }
     TQR_PH(0);
 
     // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib), one pass per half
     double c1[2][G::MF][G::JC][2];
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-        if (h == 1) { cp_async_wait<0>(); __syncwarp(); }   // half B + T block
+        mbar_wait(&sm.mbar[wq][h], (vph >> h) & 1u);
+        vph ^= 1u << h;
         const double* vh = &sm.Vst[wq][h][0][0];
 #pragma unroll
         for (int mf = 0; mf < G::MF; ++mf)
@@ -202,20 +221,6 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
             for (int j = 0; j < G::JC; ++j) c1[h][mf][j][0] = c1[h][mf][j][1] = 0.0;
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
-            if (h == 0 && nf == 0) {
-                // overlap: T block and the first part of half B behind these DMMAs
-                constexpr int TCH = IB * IB / 2;   // 16-byte chunks of the T block
-                for (int id = tid; id < TCH; id += kThreads) {
-                    const int c = id / (IB / 2), r2 = id % (IB / 2);
-                    cp_async16<CG>(&sm.Traw[c * G::LDT2 + 2 * r2], Ts + c * IB + 2 * r2);
-                }
-                stage_part<NB, W, IB, FACT, CG>(sm, Vs, ldv, 1, 0, G::NF > 1 ? QH : NQ);
-                if (G::NF == 1) cp_async_commit();
-            }
-            if (h == 0 && nf == 1) {
-                stage_part<NB, W, IB, FACT, CG>(sm, Vs, ldv, 1, QH, NQ);
-                cp_async_commit();
-            }
             if (KM && rbase + nf * 8 + 8 <= kmin) continue;  // V rows all zero (warp-uniform)
             double2 b[G::JC];
 #pragma unroll
@@ -288,6 +293,7 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
             sm.red[col * G::LDR + ib] = topv[r] + s;   // slot-0 entry (col, ib) is read above by this thread only
         }
     }
+    cp_async_wait<0>();                      // this thread's T-block chunks landed
     __syncthreads();
     TQR_PH(5);
     // ---- (3) W'^T = W^T op(T)^T on DMMA (W x IB output, 8x8 fragments spread over the warps):
@@ -328,19 +334,10 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
     //      inside the half-B loop (half A of this block is no longer read there)
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-        if (h == 1) __syncwarp();
+        if (h == 1 && next != nullptr) stage_bulk(sm, next, 0);   // half A of the next block
         const double* vh = &sm.Vst[wq][h][0][0];
 #pragma unroll
         for (int kk = 0; kk < G::HC; kk += 4) {
-            if (h == 1 && next != nullptr) {
-                if (kk == 0) {
-                    stage_part<NB, W, IB, FACT, CG>(sm, next, ldv, 0, 0, G::HC > 4 ? QH : NQ);
-                    if (G::HC <= 4) cp_async_commit();
-                } else if (kk == 4) {
-                    stage_part<NB, W, IB, FACT, CG>(sm, next, ldv, 0, QH, NQ);
-                    cp_async_commit();
-                }
-            }
             double a[G::MF];
 #pragma unroll
             for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + h * G::HC + kk + t];
@@ -354,7 +351,7 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
         }
         TQR_PH(8 + h);
     }
-    // Exit: at most one cp.async group (half A of `next`) pending.  The next call's first
+    // Exit: at most one bulk copy (half A of `next`) in flight.  The next call's first
     // barrier is preceded only by warp-private Vst traffic and red stores into slots that every
     // warp finished reading before this call's last barrier.
 }

@@ -46,7 +46,8 @@ struct Owner {
     int32_t* cols_dev = nullptr;
     double* tiles = nullptr;        // ncols * p * nb*nb
     double* T = nullptr;            // ncols * p * ib*nb
-    double* Vexp = nullptr;         // ncols * nb*nb
+    double* Vimg = nullptr;         // ncols * p * nb*nb  stage images of the reflector tiles (update-kernel operand)
+    double* Vexp = nullptr;         // ncols * nb*nb      stage image of the explicit V of each diagonal tile
     double* rb_tiles[2] = {nullptr, nullptr};
     double* rb_T[2] = {nullptr, nullptr};
     double* rb_V[2] = {nullptr, nullptr};
@@ -155,7 +156,7 @@ double flops_panel(const tqr_plan_s* h, int k) {
 void free_owner(Owner& o) {
     cudaSetDevice(o.dev);
     auto F = [](void* p) { if (p) cudaFree(p); };
-    F(o.cols_dev); F(o.tiles); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
+    F(o.cols_dev); F(o.tiles); F(o.Vimg); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
     for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref})
         for (auto e : *v) if (e) cudaEventDestroy(e);
@@ -205,6 +206,24 @@ PtrInfo classify(const void* p) {
     if (e != cudaSuccess) { cudaGetLastError(); return {Mem::Host, -1}; }
     if (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged) return {Mem::Device, at.device};
     return {Mem::Host, -1};
+}
+
+// Entry barrier of every call that reads or writes a caller buffer: the caller may have produced
+// A / B with work still queued on any stream of the device (e.g. PyTorch's current stream), and
+// the plan's streams are non-blocking, so wait for the whole device first.
+tqr_status sync_entry(tqr_plan h, const PtrInfo& pi) {
+    int prev = -1;
+    for (auto& o : h->owners) {
+        if (o.dev == prev) continue;
+        prev = o.dev;
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        CUDA_TRY(h, cudaDeviceSynchronize());
+    }
+    if (pi.kind == Mem::Device && pi.dev >= 0 && pi.dev != prev) {
+        CUDA_TRY(h, cudaSetDevice(pi.dev));
+        CUDA_TRY(h, cudaDeviceSynchronize());
+    }
+    return TQR_OK;
 }
 
 tqr_status ensure_io(tqr_plan h, Owner& o) {
@@ -415,7 +434,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
             if (cudaMalloc(ptr, elems * sizeof(double)) != cudaSuccess) { cudaGetLastError(); return false; }
             return true;
         };
-        if (!alloc(&ow.tiles, nc * p * tile) || !alloc(&ow.T, nc * p * tsz) || !alloc(&ow.Vexp, nc * tile))
+        if (!alloc(&ow.tiles, nc * p * tile) || !alloc(&ow.Vimg, nc * p * tile) || !alloc(&ow.T, nc * p * tsz) ||
+            !alloc(&ow.Vexp, nc * tile))
             return bail(fail(h, TQR_ERR_ALLOC, "tile storage allocation failed"));
         if (nc) {
             if (cudaMemset(ow.T, 0, nc * p * tsz * sizeof(double)) != cudaSuccess)
@@ -495,6 +515,7 @@ tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
     const PtrInfo pi = classify(A);
     const int64_t p = h->p, nb = h->nb, tile = nb * nb;
     h->factored = false;
+    { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
     for (auto& o : h->owners) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, cudaSetDevice(o.dev));
@@ -565,6 +586,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             const int lc = O->lidx[k];
             PanelArgs a;
             a.col = O->tiles + lc * colsz;
+            a.Vimg = O->Vimg + lc * colsz;
             a.T = O->T + lc * (int64_t)p * tsz;
             a.Vexp = O->Vexp + lc * tile;
             a.flags = O->flags;
@@ -592,7 +614,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             double *bt, *bT, *bV;
             if (root) {
                 const int lc = R.lidx[k];
-                bt = R.tiles + lc * colsz; bT = R.T + lc * (int64_t)p * tsz; bV = R.Vexp + lc * tile;
+                bt = R.Vimg + lc * colsz; bT = R.T + lc * (int64_t)p * tsz; bV = R.Vexp + lc * tile;
             } else {
                 bt = R.rb_tiles[slot]; bT = R.rb_T[slot]; bV = R.rb_V[slot];
             }
@@ -617,7 +639,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_look[k - 2], 0));
                 }
                 const int lc = O->lidx[k];
-                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_tiles[slot] + k * tile, D.dev, O->tiles + lc * colsz + k * tile,
+                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_tiles[slot] + k * tile, D.dev, O->Vimg + lc * colsz + k * tile,
                                                 O->dev, sizeof(double) * (size_t)(p - k) * tile, D.s_comm));
                 CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_T[slot] + k * tsz, D.dev, O->T + lc * (int64_t)p * tsz + k * tsz,
                                                 O->dev, sizeof(double) * (size_t)(p - k) * tsz, D.s_comm));
@@ -633,7 +655,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             UpdateArgs u;
             if (mine) {
                 const int lc = D.lidx[k];
-                u.V = D.tiles + lc * colsz; u.T = D.T + lc * (int64_t)p * tsz; u.Vexp = D.Vexp + lc * tile;
+                u.V = D.Vimg + lc * colsz; u.T = D.T + lc * (int64_t)p * tsz; u.Vexp = D.Vexp + lc * tile;
             } else {
                 const int slot = k & 1;
                 u.V = D.rb_tiles[slot]; u.T = D.rb_T[slot]; u.Vexp = D.rb_V[slot];
@@ -718,6 +740,7 @@ tqr_status tqr_store_r(tqr_plan h, void* Av, int64_t lda) {
     double* A = static_cast<double*>(Av);
     const PtrInfo pi = classify(A);
     const int64_t p = h->p, nb = h->nb, tile = nb * nb;
+    { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
     for (auto& o : h->owners) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, cudaSetDevice(o.dev));
@@ -766,7 +789,7 @@ static tqr_status apply_device(tqr_plan h, char trans, double* Bw, int64_t ldw, 
         Owner* O = h->local(h->owner_of[k]);
         const int lc = O->lidx[k];
         UpdateArgs u;
-        u.V = O->tiles + lc * colsz; u.T = O->T + lc * (int64_t)p * tsz; u.Vexp = O->Vexp + lc * tile;
+        u.V = O->Vimg + lc * colsz; u.T = O->T + lc * (int64_t)p * tsz; u.Vexp = O->Vexp + lc * tile;
         u.X = Bw; u.col_stride = (int64_t)nb * ldw; u.tile_stride = nb; u.ld = ldw;
         u.group0 = 0; u.gstride = 1; u.k = k; u.p = p; u.do_unmqr = 1;
         CUDA_TRY(h, tqr::launch_update(nb, ib, 32, u, (int)nslices, fwd, s));
@@ -805,6 +828,8 @@ tqr_status tqr_apply_qt(tqr_plan h, char trans, void* Bv, int64_t ldb, int64_t n
     CUDA_TRY(h, cudaSetDevice(dev));
     cudaStream_t s = h->owners[0].s_upd;
     double* B = static_cast<double*>(Bv);
+    st = sync_entry(h, classify(B));
+    if (st) return st;
     int64_t nsl = 0;
     st = stage_b(h, B, ldb, nrhs, &nsl, s);
     if (st) return st;
@@ -828,6 +853,8 @@ tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
     CUDA_TRY(h, cudaSetDevice(dev));
     cudaStream_t s = h->owners[0].s_upd;
     double* B = static_cast<double*>(Bv);
+    st = sync_entry(h, classify(B));
+    if (st) return st;
     int64_t nsl = 0;
     st = stage_b(h, B, ldb, nrhs, &nsl, s);
     if (st) return st;

@@ -10,7 +10,8 @@ namespace tqr {
 struct PanelArgs {
     double* col;       // the owner's tiles of column k: tile i at col + i*nb*nb (column-major nb x nb)
     double* T;         // T factors of column k: tile i at T + i*ib*nb (ib x nb, LAPACK dgeqrt layout)
-    double* Vexp;      // explicit unit-lower V of the diagonal tile (nb x nb), written by GEQRT
+    double* Vimg;      // stage images of column k's reflector tiles: tile i at Vimg + i*nb*nb (TSQRT writes)
+    double* Vexp;      // stage image of the explicit unit-lower V of the diagonal tile (GEQRT writes)
     unsigned* flags;   // p * (nb/ib) publication flags
     unsigned epoch;    // value published for this launch (monotone across launches)
     int k;             // step (tile column / diagonal tile row)
@@ -20,8 +21,8 @@ struct PanelArgs {
 // Trailing update of step k over `ngroups` column groups (UNMQR + TSMQR chain), or the
 // application of panel k's Q^T / Q to a right-hand side block (tqr_apply_qt).
 struct UpdateArgs {
-    const double* V;     // reflector tiles of panel k: tile i at V + i*nb*nb (rows k+1.. used)
-    const double* Vexp;  // explicit V of the diagonal tile
+    const double* V;     // stage images of panel k's reflector tiles: tile i at V + i*nb*nb (i > k used)
+    const double* Vexp;  // stage image of the explicit V of the diagonal tile
     const double* T;     // T factors: tile i at T + i*ib*nb
     double* X;           // target: element (tile i, r, c) of group gidx at
                          //   X + gidx*col_stride + i*tile_stride + c*ld + r
