@@ -369,3 +369,16 @@ extern "C" int tqr_probe_phases(unsigned long long* out, int reset) {
     return (int)cudaGetLastError();
 }
 #endif
+
+// Every instantiated workspace must fit the sm_100a opt-in limit of 227 KB dynamic smem per CTA.
+namespace tqr {
+constexpr size_t kMaxSmem = 232448;
+#define TQR_FITS(NB_, IB_)                                                             \
+    static_assert(sizeof(Smem<NB_, IB_, IB_, true>) <= kMaxSmem, "panel smem");        \
+    static_assert(sizeof(Smem<NB_, 8, IB_, false>) <= kMaxSmem, "update smem W=8");    \
+    static_assert(sizeof(Smem<NB_, 16, IB_, false>) <= kMaxSmem, "update smem W=16");  \
+    static_assert(sizeof(Smem<NB_, 32, IB_, false>) <= kMaxSmem, "update smem W=32");
+TQR_FITS(64, 16) TQR_FITS(64, 32) TQR_FITS(128, 16) TQR_FITS(128, 32)
+TQR_FITS(256, 16) TQR_FITS(256, 32) TQR_FITS(512, 16) TQR_FITS(512, 32)
+#undef TQR_FITS
+}  // namespace tqr

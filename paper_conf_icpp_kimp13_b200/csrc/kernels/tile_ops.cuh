@@ -76,11 +76,12 @@ struct Smem {
     double gram_pad[PADN];             // Vst..gram_pad is the contiguous Gram scratch of factor_block
     double Wsm[W * G::LDW];            // -op(T) W  (A operand of GEMM2), element (ib, col) at col*LDW + ib
     double Traw[IB * G::LDT2];         // T block s, element (r', r) at r*LDT2 + r'
+    double topsm[W * G::LDW];          // top rows X1 (IB x W), element (r, c) at c*LDW + r
     double Tsm[FACT ? IB * G::LDT : 2];   // factor_block output T(i, c) at i*LDT + c
     double Rsm[FACT ? IB * IB : 2];       // TSQRT diagonal R block (row c, col j) at c*IB + j
-    double tau[IB];
-    double wvec[IB];
-    double red1[kWarps];
+    double tau[FACT ? IB : 2];
+    double wvec[FACT ? IB : 2];
+    double red1[FACT ? kWarps : 2];
     double x0;
     uint64_t mbar[kWarps][2];          // bulk-copy completion of Vst[w][h] (outside the Gram scratch)
 };
@@ -183,26 +184,25 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
                                             const double* next, unsigned& vph) {
     using G = Geom<NB, W, IB>;
     using SM = Smem<NB, W, IB, FACT>;
-    constexpr int NR = (W * IB + kThreads - 1) / kThreads;     // reduce outputs per thread
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW;
     const int tid = threadIdx.x;
     TQR_PH0();
 
-    // ---- (0) top rows -> registers (consumed after the reduction barrier)
-    double topv[NR];
-#pragma unroll
-    for (int r = 0; r < NR; ++r) {
-        const int idx = tid + r * kThreads;
-        topv[r] = 0.0;
-        if (top && idx < W * IB) topv[r] = top[(int64_t)(idx / IB) * ldtop + (idx % IB)];
-    }
+    // ---- (0) half B of V (bulk), T block and top rows (LDGSTS group, waited before barrier 1)
     stage_bulk(sm, Vs, 1);                    // half B of this block (its buffer was read last call)
-    {   // T block -> Traw (LDGSTS group; waited before the reduction barrier)
-        constexpr int TCH = IB * IB / 2;
+    {
+        constexpr int TCH = IB * IB / 2;      // 16-byte chunks of the T block
         for (int id = tid; id < TCH; id += kThreads) {
             const int c = id / (IB / 2), r2 = id % (IB / 2);
             cp_async16<CG>(&sm.Traw[c * G::LDT2 + 2 * r2], Ts + c * IB + 2 * r2);
+        }
+        if (top) {
+            constexpr int XCH = W * IB / 2;   // 16-byte chunks of the top rows
+            for (int id = tid; id < XCH; id += kThreads) {
+                const int c = id / (IB / 2), r2 = id % (IB / 2);
+                cp_async16<true>(&sm.topsm[c * G::LDW + 2 * r2], top + (int64_t)c * ldtop + 2 * r2);
+            }
         }
         cp_async_commit();
     }
@@ -238,10 +238,11 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
         TQR_PH(1 + h);
     }
     // c1[h][mf][j] = W^T[col mf*8+g][ib h*HC + j*8 + 2t + e]
-    // ---- (2) cross-warp reduction of the 8 partials (+ top) into slot 0
+    // ---- (2) GEMM1 partials -> smem slots (8 slots, or 4 with a pairwise add for the panel)
     auto frag_ptr = [&](int slot, int h, int mf, int j) {
         return sm.red + slot * (W * G::LDR) + (mf * 8 + g) * G::LDR + h * G::HC + j * 8 + 2 * t;
     };
+    cp_async_wait<0>();                       // this thread's T-block / top-row chunks landed
     if constexpr (SM::NSLOT == 8) {
 #pragma unroll
         for (int h = 0; h < 2; ++h)
@@ -277,58 +278,51 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
         __syncthreads();
     }
     TQR_PH(4);
-#pragma unroll
-    for (int r = 0; r < NR; ++r) {
-        const int idx = tid + r * kThreads;
-        if (idx < W * IB) {
-            const int col = idx / IB, ib = idx % IB;
-            const double* rp = sm.red + col * G::LDR + ib;
-            double s = 0.0;
-            if constexpr (SM::NSLOT == 8) {
-                s = ((rp[0] + rp[W * G::LDR]) + (rp[2 * W * G::LDR] + rp[3 * W * G::LDR])) +
-                    ((rp[4 * W * G::LDR] + rp[5 * W * G::LDR]) + (rp[6 * W * G::LDR] + rp[7 * W * G::LDR]));
-            } else {
-                s = (rp[0] + rp[W * G::LDR]) + (rp[2 * W * G::LDR] + rp[3 * W * G::LDR]);
-            }
-            sm.red[col * G::LDR + ib] = topv[r] + s;   // slot-0 entry (col, ib) is read above by this thread only
-        }
-    }
-    cp_async_wait<0>();                      // this thread's T-block chunks landed
-    __syncthreads();
-    TQR_PH(5);
-    // ---- (3) W'^T = W^T op(T)^T on DMMA (W x IB output, 8x8 fragments spread over the warps):
+    // ---- (3) fused reduction + T multiply on DMMA: W'^T = (top + sum_slots P)^T op(T)^T,
     //      C[m = col][n = r] = sum_k W^T[col][k] B[k][n],  B = T (TRANS: W' = T^T W) or T^T.
-    //      Wsm = -W'.  T has explicit zeros off its triangle.
+    //      The A operand (W^T fragment) is summed from the partial slots as it is loaded; each
+    //      warp owns fragments with one column block mf so it sums that A operand once.
+    //      Wsm = -W' (GEMM2 operand); top -= W' written straight from the fragments.
     {
         constexpr int NFRAG = G::MF * G::JF;
-        for (int f = wq; f < NFRAG; f += kWarps) {
-            const int mf = f / G::JF, jf = f % G::JF;
-            double c0 = 0.0, c1v = 0.0;
+        constexpr int FPW = (NFRAG + kWarps - 1) / kWarps;   // fragments per warp (JF % FPW == 0)
+        static_assert(NFRAG <= kWarps || G::JF % FPW == 0, "fragment assignment");
+        if (wq * FPW < NFRAG) {
+            const int f0 = wq * FPW;
+            const int mf = f0 / G::JF;
+            double acc0[FPW][2], acc1[FPW][2];
+#pragma unroll
+            for (int u = 0; u < FPW; ++u) acc0[u][0] = acc0[u][1] = acc1[u][0] = acc1[u][1] = 0.0;
             const double* wa = sm.red + (mf * 8 + g) * G::LDR + t;
+            const double* ta = sm.topsm + (mf * 8 + g) * G::LDW + t;
 #pragma unroll
             for (int kk = 0; kk < IB; kk += 4) {
-                const double av = wa[kk];
-                double bv;
-                if constexpr (TRANS) bv = sm.Traw[(jf * 8 + g) * G::LDT2 + kk + t];   // T(kk+t, r)
-                else                 bv = sm.Traw[(kk + t) * G::LDT2 + jf * 8 + g];   // T(r, kk+t)
-                dmma(c0, c1v, av, bv);
+                double av = top ? ta[kk] : 0.0;
+#pragma unroll
+                for (int sl = 0; sl < SM::NSLOT; ++sl) av += wa[sl * (W * G::LDR) + kk];
+#pragma unroll
+                for (int u = 0; u < FPW; ++u) {
+                    const int jf = (f0 + u) % G::JF;
+                    double bv;
+                    if constexpr (TRANS) bv = sm.Traw[(jf * 8 + g) * G::LDT2 + kk + t];   // T(kk+t, r)
+                    else                 bv = sm.Traw[(kk + t) * G::LDT2 + jf * 8 + g];   // T(r, kk+t)
+                    if ((kk >> 2) & 1) dmma(acc1[u][0], acc1[u][1], av, bv);
+                    else               dmma(acc0[u][0], acc0[u][1], av, bv);
+                }
             }
-            st2(&sm.Wsm[(mf * 8 + g) * G::LDW + jf * 8 + 2 * t], -c0, -c1v);
+#pragma unroll
+            for (int u = 0; u < FPW; ++u) {
+                const int jf = (f0 + u) % G::JF;
+                const double w0 = acc0[u][0] + acc1[u][0], w1 = acc0[u][1] + acc1[u][1];
+                const int col = mf * 8 + g, r = jf * 8 + 2 * t;
+                st2(&sm.Wsm[col * G::LDW + r], -w0, -w1);
+                if (top) st2(top + (int64_t)col * ldtop + r, sm.topsm[col * G::LDW + r] - w0,
+                             sm.topsm[col * G::LDW + r + 1] - w1);
+            }
         }
     }
     __syncthreads();
     TQR_PH(6);
-    // top -= W'  (original top in topv, same per-thread mapping as the reduction)
-    if (top) {
-#pragma unroll
-        for (int r = 0; r < NR; ++r) {
-            const int idx = tid + r * kThreads;
-            if (idx < W * IB) {
-                const int col = idx / IB, rr = idx % IB;
-                top[(int64_t)col * ldtop + rr] = topv[r] + sm.Wsm[col * G::LDW + rr];
-            }
-        }
-    }
     TQR_PH(7);
     // ---- (4) GEMM2: X^T(col, row) += (-W'^T)(col, ib) V^T(ib, row); half A of `next` staged
     //      inside the half-B loop (half A of this block is no longer read there)
