@@ -408,10 +408,8 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                         else if (r == d) X.acc[mfc][nf][e] = beta;
                     }
             }
-            if (threadIdx.x == 0) {
-                sm.tau[c] = tau;
-                if (!GE) sm.Rsm[c * IB + c] = beta;
-            }
+            if (threadIdx.x == 0) sm.tau[c] = tau;   // R(c, c) <- beta is stored after the next barrier:
+                                                     // every thread reads x0 = R(c, c) above
             // 3. v for my rows (from the lane holding column c, same t)
             double vv[G::NF][2];
 #pragma unroll
@@ -442,6 +440,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             }
             __syncthreads();
             // 5. w_j = R(c, j) + sum_w partial ; R(c, j) -= tau w_j
+            if (!GE && threadIdx.x == 0) sm.Rsm[c * IB + c] = beta;
             if (threadIdx.x > c && threadIdx.x < IB) {
                 const int j = threadIdx.x;
                 double s = GE ? 0.0 : sm.Rsm[c * IB + j];

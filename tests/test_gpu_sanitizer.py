@@ -1,0 +1,29 @@
+"""compute-sanitizer racecheck / synccheck / memcheck over small factorizations (SURVEY sec. 5:
+race detection).  Covers the inter-CTA flag wavefront of the panel kernel, the cp.async.bulk /
+mbarrier staging and the shared-memory reductions of both kernels, apply_qt and the logical-
+device (peer-copy broadcast) path."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+
+
+@pytest.mark.parametrize("tool", ["racecheck", "synccheck", "memcheck"])
+def test_sanitizer_clean(tool):
+    out = subprocess.run([SAN, "--tool", tool, "--print-limit", "10", sys.executable,
+                          os.path.join(ROOT, "tools", "debug", "sanitize_run.py")],
+                         cwd=ROOT, capture_output=True, text=True, timeout=900)
+    text = out.stdout + out.stderr
+    assert out.returncode == 0, text[-3000:]
+    assert "ok 1024 1024 512 32" in text, text[-3000:]
+    assert ("0 errors" in text) or ("0 hazards displayed (0 errors" in text), text[-3000:]
