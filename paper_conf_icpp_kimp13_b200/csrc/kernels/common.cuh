@@ -20,6 +20,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <cstdio>
 
 namespace tqr {
 
@@ -83,6 +84,20 @@ __device__ __forceinline__ void bulk_g2s(void* smem_dst, const void* gsrc, unsig
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                  ::"r"(smem_u32(smem_dst)), "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)) : "memory");
 }
+#ifdef TQR_DEBUG_WAIT
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
+    unsigned ok = 0;
+    for (long long spins = 0; !ok; ++spins) {
+        asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+                     "selp.u32 %0, 1, 0, P;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+        if (!ok && spins == (1ll << 22)) {
+            printf("TQR_DEBUG_WAIT block %d warp %d mbarrier %p parity %u\n", blockIdx.x, threadIdx.x / 32,
+                   (void*)bar, parity);
+            __trap();
+        }
+    }
+}
+#else
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
     asm volatile(
         "{\n\t.reg .pred P;\n"
@@ -90,6 +105,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
         "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
         "@!P bra WAIT_%=;\n}" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
 }
+#endif
 
 // Inter-CTA flags (panel kernel wavefront).  Publisher: data stores, __threadfence, then a
 // release store.  Consumer: acquire spin by one thread, fence, then __syncthreads.
@@ -103,7 +119,19 @@ __device__ __forceinline__ unsigned flag_acquire(const unsigned* f) {
 }
 __device__ __forceinline__ void flag_wait_geq(const unsigned* f, unsigned v) {
     if (threadIdx.x == 0) {
+#ifdef TQR_DEBUG_WAIT
+        long long spins = 0;
+        while ((int)(flag_acquire(f) - v) < 0) {
+            __nanosleep(64);
+            if (++spins == (1ll << 24)) {
+                printf("TQR_DEBUG_WAIT block %d flag %p value %u waiting for %u\n", blockIdx.x, (const void*)f,
+                       flag_acquire(f), v);
+                __trap();
+            }
+        }
+#else
         while ((int)(flag_acquire(f) - v) < 0) __nanosleep(64);
+#endif
         __threadfence();
     }
     __syncthreads();

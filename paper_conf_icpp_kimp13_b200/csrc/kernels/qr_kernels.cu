@@ -13,63 +13,103 @@
 //                   Q^T B and Q B in tqr_apply_qt.
 //   layout kernels: column-major <-> tile-major (128-bit when aligned), R out with zeroed
 //                   lower part, and the back substitution of tqr_solve_ls (Eq. 3).
+#include <algorithm>
 #include <cstdio>
 #include "tile_ops.cuh"
 #include "../tqr_internal.h"
 
 namespace tqr {
 
+#ifdef TQR_DEBUG_WAIT
+#define TQR_TRACE(...) do { if (threadIdx.x == 0) printf(__VA_ARGS__); } while (0)
+#else
+#define TQR_TRACE(...) do {} while (0)
+#endif
+
 // ============================================================================ panel kernel
-template <int NB, int IB>
+// Grid: NBLK * S CTAs; CTA (b, u) = blockIdx.x = b*S + u owns the W = IB/S columns
+// [b*IB + u*W, b*IB + (u+1)*W) of every tile of panel k.  Per tile i, every CTA of column block b
+// applies the published reflector blocks b' < b to its columns (the chain that bounds the panel,
+// now split S ways); the block's leader (u = S-1) then gathers the IB columns and factors them.
+// Flags (release/acquire): F(i, b) = block b of tile i factored, G(i, b, u) = sub-slice (b, u) of
+// tile i updated.  A CTA waits only on lower-indexed CTAs, so in-order dispatch cannot deadlock.
+template <int NB, int IB, int W>
 __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    auto& sm = *reinterpret_cast<Smem<NB, IB, IB, true>*>(smem_raw);
+    using SA = Smem<NB, W, IB, true>;      // apply workspace (mbarriers live here)
+    using SF = Smem<NB, IB, IB, true>;     // factor workspace (same memory, used after the applies)
+    auto& sa = *reinterpret_cast<SA*>(smem_raw);
+    auto& sf = *reinterpret_cast<SF*>(smem_raw);
     using G = Geom<NB, IB, IB>;
     constexpr int NBLK = NB / IB;
-    const int b = blockIdx.x;
+    constexpr int S = IB / W;
+    const int b = blockIdx.x / S, u = blockIdx.x % S;
+    const bool leader = (u == S - 1);
     const int64_t tile = (int64_t)NB * NB;
     double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
     double* Akk = col + (int64_t)a.k * tile;
-    Slice<NB, IB, IB> X;
-    stage_init(sm);
-    unsigned vph = 0;
+    unsigned* F = a.flags;                                   // p * NBLK
+    unsigned* Gf = a.flags + (int64_t)a.p * NBLK;            // p * NBLK * S
     const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
+    unsigned vph = 0;
+    stage_init(sa);
 
     for (int i = a.k; i < a.p; ++i) {
         double* Ai = col + (int64_t)i * tile;
         double* Ti = a.T + (int64_t)i * IB * NB;
         const bool ge = (i == a.k);
-        X.load_cg(Ai + (int64_t)b * IB * NB, NB);
-        for (int bp = 0; bp < b; ++bp) {
-            flag_wait_geq(a.flags + (int64_t)i * NBLK + bp, a.epoch);
-            const double* Vb = (ge ? a.Vexp : a.Vimg + (int64_t)i * tile) + (int64_t)bp * IB * NB;
-            if (lane_id() == 0) fence_proxy_async_global();   // sibling CTA's generic stores -> bulk copy
-            stage_first(sm, Vb);
-            if (ge)
-                apply_block<NB, IB, IB, true, true, true, true>(X, sm, Vb, Ti + (int64_t)bp * IB * IB, nullptr, 0,
-                                                                bp * IB, nullptr, vph);
-            else
-                apply_block<NB, IB, IB, true, true, true, false>(X, sm, Vb, Ti + (int64_t)bp * IB * IB,
-                                                                 Akk + (int64_t)b * IB * NB + bp * IB, NB, 0,
-                                                                 nullptr, vph);
+        const int c0 = b * IB + u * W;         // first column of this sub-slice
+        if (b > 0) {
+            Slice<NB, W, IB> X;
+            X.load_cg(Ai + (int64_t)c0 * NB, NB);
+            for (int bp = 0; bp < b; ++bp) {
+                TQR_TRACE("cta %d (b%d u%d) tile %d wait F(%d)\n", blockIdx.x, b, u, i, bp);
+                flag_wait_geq(F + (int64_t)i * NBLK + bp, a.epoch);
+                const double* Vb = (ge ? a.Vexp : a.Vimg + (int64_t)i * tile) + (int64_t)bp * IB * NB;
+                if (lane_id() == 0) fence_proxy_async_global();   // sibling CTA's generic stores -> bulk copy
+                stage_first(sa, Vb);
+                if (ge)
+                    apply_block<NB, W, IB, true, true, true, true>(X, sa, Vb, Ti + (int64_t)bp * IB * IB, nullptr,
+                                                                   0, bp * IB, nullptr, vph);
+                else
+                    apply_block<NB, W, IB, true, true, true, false>(X, sa, Vb, Ti + (int64_t)bp * IB * IB,
+                                                                    Akk + (int64_t)c0 * NB + bp * IB, NB, 0,
+                                                                    nullptr, vph);
+            }
+            X.store(Ai + (int64_t)c0 * NB, NB);
         }
+        if (!leader) {
+            __threadfence();
+            __syncthreads();
+            if (threadIdx.x == 0) flag_release(Gf + ((int64_t)i * NBLK + b) * S + u, a.epoch);
+            TQR_TRACE("cta %d (b%d u%d) tile %d published G\n", blockIdx.x, b, u, i);
+            continue;
+        }
+        // ---- leader: gather the IB columns of block b and factor them
+        TQR_TRACE("cta %d (b%d u%d) tile %d leader waits G\n", blockIdx.x, b, u, i);
+        for (int up = 0; up < S - 1; ++up) flag_wait_geq(Gf + ((int64_t)i * NBLK + b) * S + up, a.epoch);
+        TQR_TRACE("cta %d (b%d u%d) tile %d leader factors\n", blockIdx.x, b, u, i);
+        __syncthreads();   // own X.store above visible to all threads
+        Slice<NB, IB, IB> Xf;
+        Xf.load_cg(Ai + (int64_t)b * IB * NB, NB);
         if (ge) {
-            factor_block<NB, IB, true>(X, sm, b * IB);
+            factor_block<NB, IB, true>(Xf, sf, b * IB);
         } else {
-            // diagonal R block of this column block: R(b*IB + c, b*IB + j), upper triangle
             for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
                 const int c = idx / IB, j = idx % IB;
-                sm.Rsm[c * IB + j] = (j >= c) ? ld_cg(Akk + (int64_t)(b * IB + j) * NB + b * IB + c) : 0.0;
+                sf.Rsm[c * IB + j] = (j >= c) ? ld_cg(Akk + (int64_t)(b * IB + j) * NB + b * IB + c) : 0.0;
             }
             __syncthreads();
-            factor_block<NB, IB, false>(X, sm, b * IB);
+            factor_block<NB, IB, false>(Xf, sf, b * IB);
         }
         // publish: reflectors (LAPACK layout in the tile), their stage image (TSQRT: V2 of tile i;
         // GEQRT: explicit unit-lower V of the diagonal tile), the T block, the R block (TSQRT)
-        X.store(Ai + (int64_t)b * IB * NB, NB);
+        // GEQRT: rows < b*IB of these columns are R rows finished by the sub-slice applies and may
+        // already be updated as TS "tops" of tile k+1 by the sub-slice CTAs: store rows >= b*IB only.
+        Xf.store_rows_from(Ai + (int64_t)b * IB * NB, NB, ge ? b * IB : 0);
         for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
             const int c = idx / IB, r = idx % IB;   // T(r, c) -> column-major block b
-            Ti[(int64_t)b * IB * IB + c * IB + r] = sm.Tsm[r * IB + c];
+            Ti[(int64_t)b * IB * IB + c * IB + r] = sf.Tsm[r * IB + c];
         }
         double* img = ge ? a.Vexp : a.Vimg + (int64_t)i * tile;
 #pragma unroll
@@ -80,7 +120,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
             for (int nf = 0; nf < G::NF; ++nf) {
                 const int rl = nf * 8 + 2 * t;         // row within this warp's rows
                 const int r = wq * G::RW + rl;
-                double v0 = X.acc[mf][nf][0], v1 = X.acc[mf][nf][1];
+                double v0 = Xf.acc[mf][nf][0], v1 = Xf.acc[mf][nf][1];
                 if (ge) {
                     v0 = (r > dc) ? v0 : (r == dc ? 1.0 : 0.0);
                     v1 = (r + 1 > dc) ? v1 : (r + 1 == dc ? 1.0 : 0.0);
@@ -91,13 +131,14 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         if (!ge) {
             for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
                 const int j = idx / IB, c = idx % IB;
-                if (c <= j) Akk[(int64_t)(b * IB + j) * NB + b * IB + c] = sm.Rsm[c * IB + j];
+                if (c <= j) Akk[(int64_t)(b * IB + j) * NB + b * IB + c] = sf.Rsm[c * IB + j];
             }
         }
         fence_proxy_async_global();
         __threadfence();
         __syncthreads();
-        if (threadIdx.x == 0) flag_release(a.flags + (int64_t)i * NBLK + b, a.epoch);
+        if (threadIdx.x == 0) flag_release(F + (int64_t)i * NBLK + b, a.epoch);
+        TQR_TRACE("cta %d (b%d u%d) tile %d published F\n", blockIdx.x, b, u, i);
     }
 }
 
@@ -231,13 +272,13 @@ __global__ void zero_diag_check_kernel(const double* __restrict__ R, int64_t ldr
 }
 
 // ============================================================================ launchers
-template <int NB, int IB>
+template <int NB, int IB, int W>
 static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s) {
-    const size_t smem = sizeof(Smem<NB, IB, IB, true>);
-    auto kern = panel_kernel<NB, IB>;
+    const size_t smem = std::max(sizeof(Smem<NB, IB, IB, true>), sizeof(Smem<NB, W, IB, true>));
+    auto kern = panel_kernel<NB, IB, W>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    kern<<<NB / IB, kThreads, smem, s>>>(a);
+    kern<<<(NB / IB) * (IB / W), kThreads, smem, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -263,15 +304,24 @@ static cudaError_t launch_update_t(const UpdateArgs& a, int nslices, bool trans,
 #define TQR_NBIB_DISPATCH(NB_, IB_, CALL)                              \
     if (nb == NB_ && ib == IB_) { return CALL; }
 
-cudaError_t launch_panel(int nb, int ib, const PanelArgs& a, cudaStream_t s) {
-    TQR_NBIB_DISPATCH(64, 16, (launch_panel_t<64, 16>(a, s)))
-    TQR_NBIB_DISPATCH(64, 32, (launch_panel_t<64, 32>(a, s)))
-    TQR_NBIB_DISPATCH(128, 16, (launch_panel_t<128, 16>(a, s)))
-    TQR_NBIB_DISPATCH(128, 32, (launch_panel_t<128, 32>(a, s)))
-    TQR_NBIB_DISPATCH(256, 16, (launch_panel_t<256, 16>(a, s)))
-    TQR_NBIB_DISPATCH(256, 32, (launch_panel_t<256, 32>(a, s)))
-    TQR_NBIB_DISPATCH(512, 16, (launch_panel_t<512, 16>(a, s)))
-    TQR_NBIB_DISPATCH(512, 32, (launch_panel_t<512, 32>(a, s)))
+template <int NB, int IB, int W>
+static cudaError_t launch_panel_chk(const PanelArgs& a, cudaStream_t s) {
+    if constexpr (W >= 8) return launch_panel_t<NB, IB, W>(a, s);
+    else return cudaErrorInvalidValue;
+}
+
+// split: sub-slices per ib column block (1, 2 or 4; W = ib / split >= 8)
+cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s) {
+#define TQR_PAN(NB_, IB_)                                                          \
+    if (nb == NB_ && ib == IB_) {                                                  \
+        if (split == 1) return launch_panel_chk<NB_, IB_, IB_>(a, s);             \
+        if (split == 2) return launch_panel_chk<NB_, IB_, IB_ / 2>(a, s);         \
+        if (split == 4) return launch_panel_chk<NB_, IB_, IB_ / 4>(a, s);         \
+        return cudaErrorInvalidValue;                                              \
+    }
+    TQR_PAN(64, 16) TQR_PAN(64, 32) TQR_PAN(128, 16) TQR_PAN(128, 32)
+    TQR_PAN(256, 16) TQR_PAN(256, 32) TQR_PAN(512, 16) TQR_PAN(512, 32)
+#undef TQR_PAN
     return cudaErrorInvalidValue;
 }
 
@@ -375,6 +425,7 @@ namespace tqr {
 constexpr size_t kMaxSmem = 232448;
 #define TQR_FITS(NB_, IB_)                                                             \
     static_assert(sizeof(Smem<NB_, IB_, IB_, true>) <= kMaxSmem, "panel smem");        \
+    static_assert(sizeof(Smem<NB_, IB_ / 2, IB_, true>) <= kMaxSmem, "panel smem S=2"); \
     static_assert(sizeof(Smem<NB_, 8, IB_, false>) <= kMaxSmem, "update smem W=8");    \
     static_assert(sizeof(Smem<NB_, 16, IB_, false>) <= kMaxSmem, "update smem W=16");  \
     static_assert(sizeof(Smem<NB_, 32, IB_, false>) <= kMaxSmem, "update smem W=32");

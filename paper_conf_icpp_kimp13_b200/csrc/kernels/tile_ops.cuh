@@ -71,6 +71,9 @@ struct Smem {
     static constexpr int NSLOT = FACT ? 4 : 8;
     static constexpr int REDN = NSLOT * W * G::LDR;
     static constexpr int PADN = (FACT && G::GRAMN > G::VSTN + REDN) ? G::GRAMN - G::VSTN - REDN : 2;
+    uint64_t mbar[kWarps][2];          // bulk-copy completion of Vst[w][h]; first member, so every
+                                       // workspace variant (panel apply W / factor IB) shares it and
+                                       // no other use ever overwrites it
     double Vst[kWarps][2][G::HC][G::RW];
     double red[REDN];
     double gram_pad[PADN];             // Vst..gram_pad is the contiguous Gram scratch of factor_block
@@ -83,7 +86,6 @@ struct Smem {
     double wvec[FACT ? IB : 2];
     double red1[FACT ? kWarps : 2];
     double x0;
-    uint64_t mbar[kWarps][2];          // bulk-copy completion of Vst[w][h] (outside the Gram scratch)
 };
 
 // ---------------------------------------------------------------- register slice I/O
@@ -114,6 +116,16 @@ struct Slice {
                 acc[mf][nf][0] = v.x;
                 acc[mf][nf][1] = v.y;
             }
+    }
+    // rows >= r0min only (r0min a multiple of 8)
+    __device__ __forceinline__ void store_rows_from(double* P, int64_t ld, int r0min) const {
+        const int g = lane_id() >> 2, t = lane_id() & 3, rw = warp_id() * G::RW;
+#pragma unroll
+        for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+            for (int nf = 0; nf < G::NF; ++nf)
+                if (rw + nf * 8 + 8 > r0min)
+                    st2(P + (int64_t)(mf * 8 + g) * ld + rw + 2 * t + nf * 8, acc[mf][nf][0], acc[mf][nf][1]);
     }
     __device__ __forceinline__ void store(double* P, int64_t ld) const {
         const int g = lane_id() >> 2, t = lane_id() & 3, r0 = warp_id() * G::RW + 2 * t;

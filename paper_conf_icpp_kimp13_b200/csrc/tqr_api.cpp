@@ -81,6 +81,7 @@ struct tqr_plan_s {
     int rank = 0, world = 1;
     bool lookahead = true, profile = false;
     int nstreams = 4;               // bulk-update streams per owner (TQR_UPDATE_STREAMS)
+    int panel_split = 1;            // sub-slice CTAs per ib column block in the panel kernel
     std::vector<Owner> owners;      // in-process: ndev entries; multi-process: 1 (this rank)
     const tqr::NcclApi* nccl = nullptr;
     ncclComm_t comm = nullptr;
@@ -385,6 +386,12 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
+    // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
+    // panel is on the critical path (few trailing columns per panel step or several owners).
+    h->panel_split = (h->q <= 32 || ndev > 1) ? 4 : 1;
+    if (ib < 32 && h->panel_split > 2) h->panel_split = 2;
+    if (const char* e = getenv("TQR_PANEL_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->panel_split = v; }
+    if (ib / h->panel_split < 8) h->panel_split = 1;
     h->owner_of.resize(h->q);
     for (int j = 0; j < h->q; ++j) h->owner_of[j] = g[j % g.size()];
 
@@ -454,7 +461,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
                 if (!alloc(&ow.rb_tiles[s], p * tile) || !alloc(&ow.rb_T[s], p * tsz) || !alloc(&ow.rb_V[s], tile))
                     return bail(fail(h, TQR_ERR_ALLOC, "receive buffer allocation failed"));
         if (nc) {
-            const size_t nfl = (size_t)p * (nb / ib);
+            const size_t nfl = (size_t)p * (nb / ib) * 5;   // F + up to 4 sub-slice flags
             if (cudaMalloc(&ow.flags, nfl * sizeof(unsigned)) != cudaSuccess ||
                 cudaMemset(ow.flags, 0, nfl * sizeof(unsigned)) != cudaSuccess)
                 return bail(fail(h, TQR_ERR_ALLOC, "flag allocation failed"));
@@ -594,7 +601,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             a.k = k;
             a.p = p;
             if (h->profile) CUDA_TRY(h, cudaEventRecord(O->tp0[k], O->s_panel));
-            CUDA_TRY(h, tqr::launch_panel(nb, ib, a, O->s_panel));
+            CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O->s_panel));
             h->launches++;
             if (h->profile) { CUDA_TRY(h, cudaEventRecord(O->tp1[k], O->s_panel)); O->tp_used[k] = 1; }
             CUDA_TRY(h, cudaEventRecord(O->ev_panel[k], O->s_panel));

@@ -12,7 +12,7 @@ struct PanelArgs {
     double* T;         // T factors of column k: tile i at T + i*ib*nb (ib x nb, LAPACK dgeqrt layout)
     double* Vimg;      // stage images of column k's reflector tiles: tile i at Vimg + i*nb*nb (TSQRT writes)
     double* Vexp;      // stage image of the explicit unit-lower V of the diagonal tile (GEQRT writes)
-    unsigned* flags;   // p * (nb/ib) publication flags
+    unsigned* flags;   // p * (nb/ib) * (1 + split) publication flags (F, then G)
     unsigned epoch;    // value published for this launch (monotone across launches)
     int k;             // step (tile column / diagonal tile row)
     int p;             // number of row tiles
@@ -35,7 +35,8 @@ struct UpdateArgs {
     int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
 };
 
-cudaError_t launch_panel(int nb, int ib, const PanelArgs& a, cudaStream_t s);
+// split = sub-slice CTAs per ib column block (1, 2, 4): grid = (nb/ib) * split
+cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s);
 // nslices CTAs; CTA b works on columns [b*w, b*w + w) counted from group0 (groups are nb wide)
 cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslices, bool trans, cudaStream_t s);
 // src column group of local column lc at src + (cols_dev ? cols[lc] : lc)*src_group_stride (ld = lda)
