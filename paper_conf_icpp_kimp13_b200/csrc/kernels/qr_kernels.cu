@@ -20,6 +20,18 @@
 
 namespace tqr {
 
+#ifdef TQR_PHASE_PROF
+// panel phases of the last column block's leader (the chain that bounds the panel):
+// g_phase[12] flag waits, [13] applies, [14] gather + factor, [15] publish
+__device__ unsigned long long g_pphase[8];
+#define TQR_PP(i) do { if (threadIdx.x == 0 && blockIdx.x == gridDim.x - 1) { long long _c = clock64(); \
+    atomicAdd(&g_pphase[i], (unsigned long long)(_c - _pp)); _pp = _c; } } while (0)
+#define TQR_PP0() long long _pp = clock64()
+#else
+#define TQR_PP(i) do {} while (0)
+#define TQR_PP0() do {} while (0)
+#endif
+
 #ifdef TQR_DEBUG_WAIT
 #define TQR_TRACE(...) do { if (threadIdx.x == 0) printf(__VA_ARGS__); } while (0)
 #else
@@ -53,6 +65,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
     unsigned vph = 0;
     stage_init(sa);
+    TQR_PP0();
 
     for (int i = a.k; i < a.p; ++i) {
         double* Ai = col + (int64_t)i * tile;
@@ -64,7 +77,9 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
             X.load_cg(Ai + (int64_t)c0 * NB, NB);
             for (int bp = 0; bp < b; ++bp) {
                 TQR_TRACE("cta %d (b%d u%d) tile %d wait F(%d)\n", blockIdx.x, b, u, i, bp);
+                TQR_PP(1);
                 flag_wait_geq(F + (int64_t)i * NBLK + bp, a.epoch);
+                TQR_PP(0);
                 const double* Vb = (ge ? a.Vexp : a.Vimg + (int64_t)i * tile) + (int64_t)bp * IB * NB;
                 if (lane_id() == 0) fence_proxy_async_global();   // sibling CTA's generic stores -> bulk copy
                 stage_first(sa, Vb);
@@ -89,6 +104,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         TQR_TRACE("cta %d (b%d u%d) tile %d leader waits G\n", blockIdx.x, b, u, i);
         for (int up = 0; up < S - 1; ++up) flag_wait_geq(Gf + ((int64_t)i * NBLK + b) * S + up, a.epoch);
         TQR_TRACE("cta %d (b%d u%d) tile %d leader factors\n", blockIdx.x, b, u, i);
+        TQR_PP(0);
         __syncthreads();   // own X.store above visible to all threads
         Slice<NB, IB, IB> Xf;
         Xf.load_cg(Ai + (int64_t)b * IB * NB, NB);
@@ -102,6 +118,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
             __syncthreads();
             factor_block<NB, IB, false>(Xf, sf, b * IB);
         }
+        TQR_PP(2);
         // publish: reflectors (LAPACK layout in the tile), their stage image (TSQRT: V2 of tile i;
         // GEQRT: explicit unit-lower V of the diagonal tile), the T block, the R block (TSQRT)
         // GEQRT: rows < b*IB of these columns are R rows finished by the sub-slice applies and may
@@ -139,6 +156,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         __syncthreads();
         if (threadIdx.x == 0) flag_release(F + (int64_t)i * NBLK + b, a.epoch);
         TQR_TRACE("cta %d (b%d u%d) tile %d published F\n", blockIdx.x, b, u, i);
+        TQR_PP(3);
     }
 }
 
@@ -412,9 +430,13 @@ size_t update_smem_bytes(int nb, int ib, int w) {
 #ifdef TQR_PHASE_PROF
 extern "C" int tqr_probe_phases(unsigned long long* out, int reset) {
     cudaMemcpyFromSymbol(out, tqr::g_phase, sizeof(unsigned long long) * 16);
+    cudaMemcpyFromSymbol(out + 16, tqr::g_pphase, sizeof(unsigned long long) * 8);
+    cudaMemcpyFromSymbol(out + 24, tqr::g_fphase, sizeof(unsigned long long) * 4);
     if (reset) {
         unsigned long long z[16] = {0};
         cudaMemcpyToSymbol(tqr::g_phase, z, sizeof(z));
+        cudaMemcpyToSymbol(tqr::g_pphase, z, sizeof(unsigned long long) * 8);
+        cudaMemcpyToSymbol(tqr::g_fphase, z, sizeof(unsigned long long) * 4);
     }
     return (int)cudaGetLastError();
 }

@@ -28,7 +28,13 @@ __device__ unsigned long long g_phase[16];
 #define TQR_PH(i) do { if ((threadIdx.x & 255) == 0) { long long _c = clock64(); \
     atomicAdd(&g_phase[i], (unsigned long long)(_c - _ph)); _ph = _c; } } while (0)
 #define TQR_PH0() long long _ph = clock64()
+__device__ unsigned long long g_fphase[4];
+#define TQR_FP(i) do { if (threadIdx.x == 0 && blockIdx.x == gridDim.x - 1) { long long _c = clock64(); \
+    atomicAdd(&g_fphase[i], (unsigned long long)(_c - _fp)); _fp = _c; } } while (0)
+#define TQR_FP0() long long _fp = clock64()
 #else
+#define TQR_FP(i) do {} while (0)
+#define TQR_FP0() do {} while (0)
 #define TQR_PH(i) do {} while (0)
 #define TQR_PH0() do {} while (0)
 #endif
@@ -373,6 +379,16 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
     using G = Geom<NB, IB, IB>;
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW + 2 * t;   // row of acc[.][nf][e] = rbase + nf*8 + e
+    // One barrier per column: each warp publishes, for column c, the partial ||x_below||^2, the
+    // unscaled dots x^T a_j of every column j of the block and (GEQRT) the row-d entries a_dj;
+    // after the barrier every thread forms beta, tau, scale = 1/(x0 - beta) and
+    // w_j = a_dj (GEQRT) or R(c, j) (TSQRT) + scale * sum_w (x^T a_j)_w itself (v = scale x).
+    constexpr int FBW = 2 * IB + 2;          // per-warp record: dots[IB], diag row[IB], ||x||^2
+    double* fb = sm.red;                      // [2][kWarps][FBW] (double-buffered by column parity)
+    double* Rout = sm.topsm;                  // TSQRT: R rows written as they are finished
+    static_assert(2 * kWarps * FBW <= Smem<NB, IB, IB, true>::REDN, "factor record buffer");
+    static_assert(IB * IB <= IB * G::LDW, "Rout buffer");
+    TQR_FP0();
 
 #pragma unroll
     for (int mfc = 0; mfc < G::MF; ++mfc) {
@@ -380,28 +396,62 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
         for (int gc = 0; gc < 8; ++gc) {
             const int c = mfc * 8 + gc;
             const int d = dbase + c;
-            const bool mycol = (g == gc);
-            // 1. ||x_below||^2
+            double* fbp = fb + (c & 1) * (kWarps * FBW);
+            // 1. x = column c on my rows (from the lane holding it, same t), masked to rows > d (GEQRT)
+            double xv[G::NF][2];
+#pragma unroll
+            for (int nf = 0; nf < G::NF; ++nf)
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    const double x = __shfl_sync(0xffffffffu, X.acc[mfc][nf][e], gc * 4 + t);
+                    const int r = rbase + nf * 8 + e;
+                    xv[nf][e] = (!GE || r > d) ? x : 0.0;
+                }
             double ss = 0.0;
-            if (mycol) {
+            if (g == 0) {
+#pragma unroll
+                for (int nf = 0; nf < G::NF; ++nf) ss += xv[nf][0] * xv[nf][0] + xv[nf][1] * xv[nf][1];
+            }
+            double pd[G::MF], p0[G::MF];
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf) {
+                double sdot = 0.0, sdiag = 0.0;
 #pragma unroll
                 for (int nf = 0; nf < G::NF; ++nf)
 #pragma unroll
                     for (int e = 0; e < 2; ++e) {
-                        const int r = rbase + nf * 8 + e;
-                        const double x = X.acc[mfc][nf][e];
-                        if (!GE || r > d) ss += x * x;
-                        if (GE && r == d) sm.x0 = x;
+                        sdot += xv[nf][e] * X.acc[mf][nf][e];
+                        if (GE && rbase + nf * 8 + e == d) sdiag = X.acc[mf][nf][e];
                     }
+                sdot += __shfl_xor_sync(0xffffffffu, sdot, 1);
+                sdot += __shfl_xor_sync(0xffffffffu, sdot, 2);
+                pd[mf] = sdot;
+                if (GE) {
+                    sdiag += __shfl_xor_sync(0xffffffffu, sdiag, 1);
+                    sdiag += __shfl_xor_sync(0xffffffffu, sdiag, 2);
+                }
+                p0[mf] = sdiag;
             }
             ss += __shfl_xor_sync(0xffffffffu, ss, 1);
             ss += __shfl_xor_sync(0xffffffffu, ss, 2);
-            if (lane == gc * 4) sm.red1[wq] = ss;
-            __syncthreads();
-            double xn2 = 0.0;
+            if (t == 0) {
+                double* rec = fbp + wq * FBW;
 #pragma unroll
-            for (int w = 0; w < kWarps; ++w) xn2 += sm.red1[w];
-            const double x0 = GE ? sm.x0 : sm.Rsm[c * IB + c];
+                for (int mf = 0; mf < G::MF; ++mf) {
+                    rec[mf * 8 + g] = pd[mf];
+                    if (GE) rec[IB + mf * 8 + g] = p0[mf];
+                }
+                if (g == 0) rec[2 * IB] = ss;
+            }
+            __syncthreads();
+            // 2. reflector (dlarfg convention, readings Q1/Q4): beta = -sgn(x0) ||(x0, x)||
+            double xn2 = 0.0, x0 = 0.0;
+#pragma unroll
+            for (int w = 0; w < kWarps; ++w) {
+                xn2 += fbp[w * FBW + 2 * IB];
+                if (GE) x0 += fbp[w * FBW + IB + c];
+            }
+            if (!GE) x0 = sm.Rsm[c * IB + c];
             double beta = x0, tau = 0.0, scale = 0.0;
             if (xn2 > 0.0) {
                 const double nrm = sqrt(x0 * x0 + xn2);
@@ -409,8 +459,37 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 tau = (beta - x0) / beta;
                 scale = 1.0 / (x0 - beta);
             }
-            // 2. v = x / (x0 - beta) below the diagonal; diagonal <- beta
-            if (mycol) {
+            // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = scale x (+ e_d)
+            double tw[G::MF];
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf) {
+                const int j = mf * 8 + g;
+                tw[mf] = 0.0;
+                if (j > c) {
+                    double dsum = 0.0, base = 0.0;
+#pragma unroll
+                    for (int w = 0; w < kWarps; ++w) {
+                        dsum += fbp[w * FBW + j];
+                        if (GE) base += fbp[w * FBW + IB + j];
+                    }
+                    if (!GE) base = sm.Rsm[c * IB + j];
+                    const double wj = base + scale * dsum;
+                    tw[mf] = tau * wj;
+                    if (!GE && wq == 0 && t == 0) Rout[c * IB + j] = base - tau * wj;
+                }
+            }
+#pragma unroll
+            for (int mf = 0; mf < G::MF; ++mf) {
+#pragma unroll
+                for (int nf = 0; nf < G::NF; ++nf)
+#pragma unroll
+                    for (int e = 0; e < 2; ++e) {
+                        const double v = scale * xv[nf][e] + ((GE && rbase + nf * 8 + e == d) ? 1.0 : 0.0);
+                        X.acc[mf][nf][e] -= tw[mf] * v;
+                    }
+            }
+            // column c itself: v below the diagonal, beta on it
+            if (g == gc) {
 #pragma unroll
                 for (int nf = 0; nf < G::NF; ++nf)
 #pragma unroll
@@ -420,63 +499,22 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                         else if (r == d) X.acc[mfc][nf][e] = beta;
                     }
             }
-            if (threadIdx.x == 0) sm.tau[c] = tau;   // R(c, c) <- beta is stored after the next barrier:
-                                                     // every thread reads x0 = R(c, c) above
-            // 3. v for my rows (from the lane holding column c, same t)
-            double vv[G::NF][2];
-#pragma unroll
-            for (int nf = 0; nf < G::NF; ++nf)
-#pragma unroll
-                for (int e = 0; e < 2; ++e) {
-                    const double x = __shfl_sync(0xffffffffu, X.acc[mfc][nf][e], gc * 4 + t);
-                    const int r = rbase + nf * 8 + e;
-                    vv[nf][e] = GE ? ((r > d) ? x : (r == d ? 1.0 : 0.0)) : x;
-                }
-            // 4. partial dots v^T X(:, j) for my columns j > c
-            double pd[G::MF];
-#pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) {
-                double s = 0.0;
-                if (mf * 8 + g > c) {
-#pragma unroll
-                    for (int nf = 0; nf < G::NF; ++nf) s += vv[nf][0] * X.acc[mf][nf][0] + vv[nf][1] * X.acc[mf][nf][1];
-                }
-                s += __shfl_xor_sync(0xffffffffu, s, 1);
-                s += __shfl_xor_sync(0xffffffffu, s, 2);
-                pd[mf] = s;
-            }
-            if (t == 0) {
-#pragma unroll
-                for (int mf = 0; mf < G::MF; ++mf)
-                    if (mf * 8 + g > c) sm.red[wq * IB + mf * 8 + g] = pd[mf];
-            }
-            __syncthreads();
-            // 5. w_j = R(c, j) + sum_w partial ; R(c, j) -= tau w_j
-            if (!GE && threadIdx.x == 0) sm.Rsm[c * IB + c] = beta;
-            if (threadIdx.x > c && threadIdx.x < IB) {
-                const int j = threadIdx.x;
-                double s = GE ? 0.0 : sm.Rsm[c * IB + j];
-#pragma unroll
-                for (int w = 0; w < kWarps; ++w) s += sm.red[w * IB + j];
-                sm.wvec[j] = s;
-                if (!GE) sm.Rsm[c * IB + j] -= tau * s;
-            }
-            __syncthreads();
-            // 6. X(:, j) -= tau v w_j
-#pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) {
-                if (mf * 8 + g > c) {
-                    const double tw = tau * sm.wvec[mf * 8 + g];
-#pragma unroll
-                    for (int nf = 0; nf < G::NF; ++nf) {
-                        X.acc[mf][nf][0] -= tw * vv[nf][0];
-                        X.acc[mf][nf][1] -= tw * vv[nf][1];
-                    }
-                }
+            if (threadIdx.x == 0) {
+                sm.tau[c] = tau;
+                if (!GE) Rout[c * IB + c] = beta;
             }
         }
     }
+    if (!GE) {   // finished R rows -> Rsm (upper triangle)
+        __syncthreads();
+        for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+            const int c = idx / IB, j = idx % IB;
+            if (j >= c) sm.Rsm[c * IB + j] = Rout[c * IB + j];
+        }
+    }
+    __syncthreads();
 
+    TQR_FP(0);
     // ---- T factor: Gram G = V^T V (strict upper part used), DMMA on register fragments
     {
         double gacc[G::MF][G::MF][2];
@@ -521,6 +559,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             sm.Wsm[cp * G::LDW + c] = s;   // Gram(c', c)
         }
         __syncthreads();
+        TQR_FP(1);
         // forward dlarft recurrence by warp 0: T(c,c) = tau_c; T(0:c, c) = -tau_c T(0:c,0:c) G(0:c, c)
         if (wq == 0) {
             for (int i = lane; i < IB * IB; i += 32) sm.Tsm[i] = 0.0;
@@ -538,6 +577,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             }
         }
         __syncthreads();
+        TQR_FP(2);
     }
 }
 

@@ -14,7 +14,7 @@ m, n, nb, ib, seed = CONFIGS[cfg]
 g = torch.Generator(device="cuda").manual_seed(seed)
 A = torch.randn((n, m), dtype=torch.float64, device="cuda", generator=g).t()
 R = torch.empty((n, m), dtype=torch.float64, device="cuda").t()
-buf = (ctypes.c_ulonglong * 16)()
+buf = (ctypes.c_ulonglong * 28)()
 with tqr.Plan(m, n, nb, ib) as p:
     p.load(A); p.factor_tiles(); p.store_r(R)
     L.tqr_probe_phases(buf, 1)
@@ -26,3 +26,12 @@ names = ["T cp.async+top ld", "GEMM1 half A", "GEMM1 half B", "stage1 st+sync", 
 tot = sum(buf[i] for i in range(12))
 for i, nm in enumerate(names):
     print("%-20s %6.2f%%" % (nm, 100.0 * buf[i] / tot))
+
+pt = sum(buf[16 + i] for i in range(4))
+if pt:
+    print("panel last-leader chain:", ", ".join("%s %.1f%%" % (nm, 100.0 * buf[16 + i] / pt) for i, nm in
+          enumerate(["flag waits", "applies", "gather+factor", "publish"])), "total Mcycles %.1f" % (pt / 1e6))
+ft = sum(buf[24 + i] for i in range(3))
+if ft:
+    print("factor_block (last CTA): columns %.1f Mcyc, Gram %.1f Mcyc, dlarft recurrence %.1f Mcyc" %
+          tuple(buf[24 + i] / 1e6 for i in range(3)))
