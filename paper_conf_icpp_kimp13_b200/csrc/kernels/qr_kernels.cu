@@ -39,12 +39,13 @@ __device__ unsigned long long g_pphase[8];
 #endif
 
 // ============================================================================ panel kernel
-// Grid: NBLK * S CTAs; CTA (b, u) = blockIdx.x = b*S + u owns the W = IB/S columns
-// [b*IB + u*W, b*IB + (u+1)*W) of every tile of panel k.  Per tile i, every CTA of column block b
-// applies the published reflector blocks b' < b to its columns (the chain that bounds the panel,
-// now split S ways); the block's leader (u = S-1) then gathers the IB columns and factors them.
-// Flags (release/acquire): F(i, b) = block b of tile i factored, G(i, b, u) = sub-slice (b, u) of
-// tile i updated.  A CTA waits only on lower-indexed CTAs, so in-order dispatch cannot deadlock.
+// Grid: NBLK * (S + 1) CTAs.  For column block b: S "apply" CTAs (u = 0..S-1) own the W = IB/S
+// columns [b*IB + u*W, b*IB + (u+1)*W) of every tile of panel k and apply the published
+// reflector blocks b' < b of tile i to them (the chain that bounds the panel, split S ways); the
+// "factor" CTA (u = S) gathers the IB columns and factors them while the apply CTAs already
+// continue with tile i+1.  Flags (release/acquire): F(i, b) = block b of tile i factored,
+// G(i, b, u) = sub-slice (b, u) of tile i updated.  CTA index b*(S+1) + u: a CTA waits only on
+// lower-indexed CTAs, so in-order dispatch cannot deadlock.
 template <int NB, int IB, int W>
 __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -55,8 +56,8 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     using G = Geom<NB, IB, IB>;
     constexpr int NBLK = NB / IB;
     constexpr int S = IB / W;
-    const int b = blockIdx.x / S, u = blockIdx.x % S;
-    const bool leader = (u == S - 1);
+    const int b = blockIdx.x / (S + 1), u = blockIdx.x % (S + 1);
+    const bool leader = (u == S);              // the factor CTA of block b
     const int64_t tile = (int64_t)NB * NB;
     double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
     double* Akk = col + (int64_t)a.k * tile;
@@ -72,7 +73,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         double* Ti = a.T + (int64_t)i * IB * NB;
         const bool ge = (i == a.k);
         const int c0 = b * IB + u * W;         // first column of this sub-slice
-        if (b > 0) {
+        if (!leader && b > 0) {
             Slice<NB, W, IB> X;
             X.load_cg(Ai + (int64_t)c0 * NB, NB);
             for (int bp = 0; bp < b; ++bp) {
@@ -94,18 +95,20 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
             X.store(Ai + (int64_t)c0 * NB, NB);
         }
         if (!leader) {
-            __threadfence();
-            __syncthreads();
-            if (threadIdx.x == 0) flag_release(Gf + ((int64_t)i * NBLK + b) * S + u, a.epoch);
-            TQR_TRACE("cta %d (b%d u%d) tile %d published G\n", blockIdx.x, b, u, i);
+            if (b > 0) {
+                __threadfence();
+                __syncthreads();
+                if (threadIdx.x == 0) flag_release(Gf + ((int64_t)i * NBLK + b) * S + u, a.epoch);
+                TQR_TRACE("cta %d (b%d u%d) tile %d published G\n", blockIdx.x, b, u, i);
+            }
             continue;
         }
         // ---- leader: gather the IB columns of block b and factor them
         TQR_TRACE("cta %d (b%d u%d) tile %d leader waits G\n", blockIdx.x, b, u, i);
-        for (int up = 0; up < S - 1; ++up) flag_wait_geq(Gf + ((int64_t)i * NBLK + b) * S + up, a.epoch);
+        if (b > 0)
+            for (int up = 0; up < S; ++up) flag_wait_geq(Gf + ((int64_t)i * NBLK + b) * S + up, a.epoch);
         TQR_TRACE("cta %d (b%d u%d) tile %d leader factors\n", blockIdx.x, b, u, i);
         TQR_PP(0);
-        __syncthreads();   // own X.store above visible to all threads
         Slice<NB, IB, IB> Xf;
         Xf.load_cg(Ai + (int64_t)b * IB * NB, NB);
         if (ge) {
@@ -124,10 +127,6 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         // GEQRT: rows < b*IB of these columns are R rows finished by the sub-slice applies and may
         // already be updated as TS "tops" of tile k+1 by the sub-slice CTAs: store rows >= b*IB only.
         Xf.store_rows_from(Ai + (int64_t)b * IB * NB, NB, ge ? b * IB : 0);
-        for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
-            const int c = idx / IB, r = idx % IB;   // T(r, c) -> column-major block b
-            Ti[(int64_t)b * IB * IB + c * IB + r] = sf.Tsm[r * IB + c];
-        }
         double* img = ge ? a.Vexp : a.Vimg + (int64_t)i * tile;
 #pragma unroll
         for (int mf = 0; mf < IB / 8; ++mf) {
@@ -150,6 +149,11 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
                 const int j = idx / IB, c = idx % IB;
                 if (c <= j) Akk[(int64_t)(b * IB + j) * NB + b * IB + c] = sf.Rsm[c * IB + j];
             }
+        }
+        build_T<NB, IB>(sf);
+        for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+            const int c = idx / IB, r = idx % IB;   // T(r, c) -> column-major block b
+            Ti[(int64_t)b * IB * IB + c * IB + r] = sf.Tsm[r * IB + c];
         }
         fence_proxy_async_global();
         __threadfence();
@@ -296,7 +300,7 @@ static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s) {
     auto kern = panel_kernel<NB, IB, W>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    kern<<<(NB / IB) * (IB / W), kThreads, smem, s>>>(a);
+    kern<<<(NB / IB) * (IB / W + 1), kThreads, smem, s>>>(a);
     return cudaGetLastError();
 }
 

@@ -372,7 +372,8 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
 // X holds W = IB columns.  GEQRT mode (GE=true): column c's diagonal row is d = dbase + c,
 // rows < d are R (kept), rows > d become v (unit v_d implied, stored beta at row d).
 // TSQRT mode (GE=false): the top is sm.Rsm (IB x IB upper triangle, row c is R(dbase+c, :));
-// all NB rows of X are the dense V2 part.  On exit: X = reflectors, sm.tau, sm.Tsm holds the
+// all NB rows of X are the dense V2 part.  On exit: X = reflectors, sm.tau, sm.Wsm = Gram V^T V;
+// build_T then forms the
 // IB x IB T factor as Tsm[i*LDT + c] = T(i, c) (upper triangle, zeros below).
 template <int NB, int IB, bool GE>
 __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, IB, true>& sm, int dbase) {
@@ -456,8 +457,8 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             if (xn2 > 0.0) {
                 const double nrm = sqrt(x0 * x0 + xn2);
                 beta = (x0 < 0.0) ? nrm : -nrm;          // beta = -sgn(x0) ||x||, sgn(0)=+1
-                tau = (beta - x0) / beta;
-                scale = 1.0 / (x0 - beta);
+                tau = (beta - x0) / beta;                  // correctly rounded: tau ||v||^2 = 2 decides
+                scale = 1.0 / (x0 - beta);                 // the orthogonality of I - tau v v^T
             }
             // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = scale x (+ e_d)
             double tw[G::MF];
@@ -560,25 +561,36 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
         }
         __syncthreads();
         TQR_FP(1);
-        // forward dlarft recurrence by warp 0: T(c,c) = tau_c; T(0:c, c) = -tau_c T(0:c,0:c) G(0:c, c)
-        if (wq == 0) {
-            for (int i = lane; i < IB * IB; i += 32) sm.Tsm[i] = 0.0;
-            __syncwarp();
-            for (int c = 0; c < IB; ++c) {
-                const double tc = sm.tau[c];
-                double s = 0.0;
-                if (lane < c) {
-                    for (int l = lane; l < c; ++l) s += sm.Tsm[lane * G::LDT + l] * sm.Wsm[l * G::LDW + c];
-                }
-                __syncwarp();
-                if (lane < c) sm.Tsm[lane * G::LDT + c] = -tc * s;
-                if (lane == 0) sm.Tsm[c * G::LDT + c] = tc;
-                __syncwarp();
-            }
-        }
-        __syncthreads();
-        TQR_FP(2);
+        // Gram in sm.Wsm; T is built by build_T (after the caller has stored X, freeing registers)
     }
+}
+
+// Forward dlarft recurrence T(c,c) = tau_c, T(0:c, c) = -tau_c T(0:c, 0:c) G(0:c, c), one row per
+// lane of warp 0 held in registers: row i only needs its own earlier entries, so the 32 rows run
+// independently with broadcast reads of the Gram matrix (no inter-lane traffic, no barriers).
+template <int NB, int IB>
+__device__ __forceinline__ void build_T(Smem<NB, IB, IB, true>& sm) {
+    using G = Geom<NB, IB, IB>;
+    TQR_FP0();
+    if (warp_id() == 0 && lane_id() < IB) {
+        const int i = lane_id();
+        double trow[IB];
+#pragma unroll
+        for (int c = 0; c < IB; ++c) {
+            double s0 = 0.0, s1 = 0.0;
+#pragma unroll
+            for (int l = 0; l < c; ++l) {
+                const double gl = sm.Wsm[l * G::LDW + c];
+                if (l & 1) s1 += trow[l] * gl; else s0 += trow[l] * gl;
+            }
+            const double tc = sm.tau[c];
+            trow[c] = (i < c) ? -tc * (s0 + s1) : (i == c ? tc : 0.0);
+        }
+#pragma unroll
+        for (int c = 0; c < IB; ++c) sm.Tsm[i * G::LDT + c] = trow[c];
+    }
+    __syncthreads();
+    TQR_FP(2);
 }
 
 }  // namespace tqr

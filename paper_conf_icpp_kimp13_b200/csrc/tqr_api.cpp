@@ -388,7 +388,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
     // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
     // panel is on the critical path (few trailing columns per panel step or several owners).
-    h->panel_split = (h->q <= 32 || ndev > 1) ? 4 : 1;
+    h->panel_split = (h->q <= 4) ? 4 : 2;   // measured: 4 for tall / few columns, 2 otherwise
     if (ib < 32 && h->panel_split > 2) h->panel_split = 2;
     if (const char* e = getenv("TQR_PANEL_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->panel_split = v; }
     if (ib / h->panel_split < 8) h->panel_split = 1;

@@ -35,7 +35,7 @@ struct UpdateArgs {
     int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
 };
 
-// split = sub-slice CTAs per ib column block (1, 2, 4): grid = (nb/ib) * split
+// split = apply CTAs per ib column block (1, 2, 4): grid = (nb/ib) * (split + 1)
 cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s);
 // nslices CTAs; CTA b works on columns [b*w, b*w + w) counted from group0 (groups are nb wide)
 cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslices, bool trans, cudaStream_t s);
