@@ -70,7 +70,10 @@ typedef struct {
 
 /*
  * Create a plan for the QR factorisation of an m x n matrix.
- *   m, n      : matrix size, m >= n >= 1; this build needs m % nb == 0 and n % nb == 0.
+ *   m, n      : matrix size, m >= n >= 1.  Any sizes: the tile grid is p = ceil(m/nb) x
+ *               q = ceil(n/nb) and the ragged tails are zero-padded inside the plan (a zero
+ *               padded column gets tau = 0 and padded rows stay zero, so R(0:n,0:n) and
+ *               Q = diag(Q_m, I) restricted to the caller's m rows are unchanged).
  *   nb        : tile size (square tiles); supported 64, 128, 256, 512.
  *   ib        : inner blocking of the compact-WY T factors; 1 <= ib <= nb, nb % ib == 0;
  *               supported 16, 32.

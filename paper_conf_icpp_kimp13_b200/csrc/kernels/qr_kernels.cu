@@ -15,6 +15,8 @@
 //                   lower part, and the back substitution of tqr_solve_ls (Eq. 3).
 #include <algorithm>
 #include <cstdio>
+#include <cstring>
+#include <type_traits>
 #include "tile_ops.cuh"
 #include "../tqr_internal.h"
 
@@ -218,55 +220,69 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
 }
 
 // ============================================================================ layout kernels
-// a1: column-major source -> tile-major column storage.  Source column group of local column
-// lc starts at src + cols[lc]*src_group_stride (ld = lda); destination tile i of local column
-// lc at dst + lc*dst_col_stride + i*nb*nb, element (r, c) at + c*nb + r.  blockIdx.x = chunk*nb
-// + c, blockIdx.y = lc.  128-bit (double2) when lda and the pointer are 16-byte aligned: a warp
-// moves 512 contiguous bytes per instruction on both sides.
-__global__ void to_tiles_kernel(const double* __restrict__ src, int64_t lda, int64_t src_group_stride,
-                                double* __restrict__ dst, const int32_t* __restrict__ cols,
-                                int64_t dst_col_stride, int nb, int p, int vec2) {
-    const int lc = blockIdx.y;
-    const int c = blockIdx.x % nb;
-    const int chunk = blockIdx.x / nb, nchunk = gridDim.x / nb;
-    const double* s = src + (int64_t)(cols ? cols[lc] : lc) * src_group_stride + (int64_t)c * lda;
-    double* d = dst + (int64_t)lc * dst_col_stride + (int64_t)c * nb;
-    const int64_t tile = (int64_t)nb * nb;
-    const int64_t m = (int64_t)p * nb;
-    if (vec2) {
-        for (int64_t r = 2 * ((int64_t)chunk * blockDim.x + threadIdx.x); r < m; r += 2 * (int64_t)nchunk * blockDim.x) {
-            const double2 v = __ldcs(reinterpret_cast<const double2*>(s + r));
-            *reinterpret_cast<double2*>(d + (r / nb) * tile + (r % nb)) = v;
-        }
-    } else {
-        for (int64_t r = (int64_t)chunk * blockDim.x + threadIdx.x; r < m; r += (int64_t)nchunk * blockDim.x)
-            d[(r / nb) * tile + (r % nb)] = s[r];
-    }
-}
-
-// a8: tile-major -> column-major rows [0, m_rows): R on and above the diagonal, 0 below.
-__global__ void from_tiles_kernel(double* __restrict__ dst, int64_t lda, int64_t dst_group_stride,
-                                  const double* __restrict__ src, const int32_t* __restrict__ cols,
-                                  int64_t src_col_stride, int nb, int64_t m_rows, int local_dst, int vec2) {
+// a1: column-major source -> tile-major column storage, zero-padded to whole tiles (rows >= m_valid
+// and global columns >= n_valid are written as 0: a padded zero column gets tau = 0 and padded zero
+// rows stay zero under every reflector, so Q = diag(Q_m, I) and R(0:n, 0:n) is unchanged).
+// Source group of local column lc at src + (local_src ? lc : cols[lc])*src_group_stride (ld = lda);
+// destination tile i of local column lc at dst + lc*dst_col_stride + i*nb*nb, element (r, c) at
+// + c*nb + r.  blockIdx.x = chunk*nb + c, blockIdx.y = lc.  VEC elements per 16-byte access when
+// lda, the group stride, m_valid and the pointer allow it: a warp moves 512 contiguous bytes per
+// instruction on both sides.
+template <class T, int VEC>
+__global__ void to_tiles_kernel(const T* __restrict__ src, int64_t lda, int64_t src_group_stride,
+                                T* __restrict__ dst, const int32_t* __restrict__ cols, int local_src,
+                                int64_t dst_col_stride, int nb, int p, int64_t m_valid, int64_t n_valid) {
+    using V = typename std::conditional<VEC == 1, T, typename std::conditional<sizeof(T) == 8, double2, float4>::type>::type;
     const int lc = blockIdx.y;
     const int c = blockIdx.x % nb;
     const int chunk = blockIdx.x / nb, nchunk = gridDim.x / nb;
     const int64_t gcol = (int64_t)cols[lc] * nb + c;
-    double* d = dst + (int64_t)(local_dst ? lc : cols[lc]) * dst_group_stride + (int64_t)c * lda;
-    const double* s = src + (int64_t)lc * src_col_stride + (int64_t)c * nb;
+    const bool colv = gcol < n_valid;
+    const T* s = src + (int64_t)(local_src ? lc : cols[lc]) * src_group_stride + (int64_t)c * lda;
+    T* d = dst + (int64_t)lc * dst_col_stride + (int64_t)c * nb;
     const int64_t tile = (int64_t)nb * nb;
-    if (vec2) {
-        for (int64_t r = 2 * ((int64_t)chunk * blockDim.x + threadIdx.x); r < m_rows; r += 2 * (int64_t)nchunk * blockDim.x) {
-            double2 v = make_double2(0.0, 0.0);
-            if (r <= gcol) {
-                v = *reinterpret_cast<const double2*>(s + (r / nb) * tile + (r % nb));
-                if (r + 1 > gcol) v.y = 0.0;
+    const int64_t m = (int64_t)p * nb;
+    for (int64_t r = VEC * ((int64_t)chunk * blockDim.x + threadIdx.x); r < m; r += VEC * (int64_t)nchunk * blockDim.x) {
+        V v{};
+        if (colv && r < m_valid) v = __ldcs(reinterpret_cast<const V*>(s + r));
+        *reinterpret_cast<V*>(d + (r / nb) * tile + (r % nb)) = v;
+    }
+}
+
+// a8: tile-major -> column-major rows [0, m_rows) of the global columns < n_valid: R on and above
+// the diagonal, 0 below.  Destination group at dst + (local_dst ? lc : cols[lc])*dst_group_stride.
+template <class T, int VEC>
+__global__ void from_tiles_kernel(T* __restrict__ dst, int64_t lda, int64_t dst_group_stride,
+                                  const T* __restrict__ src, const int32_t* __restrict__ cols,
+                                  int64_t src_col_stride, int nb, int64_t m_rows, int64_t n_valid, int local_dst) {
+    const int lc = blockIdx.y;
+    const int c = blockIdx.x % nb;
+    const int chunk = blockIdx.x / nb, nchunk = gridDim.x / nb;
+    const int64_t gcol = (int64_t)cols[lc] * nb + c;
+    if (gcol >= n_valid) return;
+    T* d = dst + (int64_t)(local_dst ? lc : cols[lc]) * dst_group_stride + (int64_t)c * lda;
+    const T* s = src + (int64_t)lc * src_col_stride + (int64_t)c * nb;
+    const int64_t tile = (int64_t)nb * nb;
+    for (int64_t r = VEC * ((int64_t)chunk * blockDim.x + threadIdx.x); r < m_rows; r += VEC * (int64_t)nchunk * blockDim.x) {
+        T v[VEC];
+#pragma unroll
+        for (int e = 0; e < VEC; ++e) v[e] = T(0);
+        if (r <= gcol) {
+            if constexpr (VEC == 1) {
+                v[0] = s[(r / nb) * tile + (r % nb)];
+            } else {
+                const T* sp = s + (r / nb) * tile + (r % nb);
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) v[e] = (r + e <= gcol) ? sp[e] : T(0);
             }
-            __stcs(reinterpret_cast<double2*>(d + r), v);
         }
-    } else {
-        for (int64_t r = (int64_t)chunk * blockDim.x + threadIdx.x; r < m_rows; r += (int64_t)nchunk * blockDim.x)
-            d[r] = (r <= gcol) ? s[(r / nb) * tile + (r % nb)] : 0.0;
+        if constexpr (VEC == 1) {
+            d[r] = v[0];
+        } else if constexpr (sizeof(T) == 8) {
+            __stcs(reinterpret_cast<double2*>(d + r), make_double2(v[0], v[1]));
+        } else {
+            __stcs(reinterpret_cast<float4*>(d + r), make_float4(v[0], v[1], v[2], v[3]));
+        }
     }
 }
 
@@ -368,35 +384,56 @@ cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslice
     return cudaErrorInvalidValue;
 }
 
-static int layout_chunks(int64_t m, int vec2, int threads) {
-    int64_t chunks = (m / (vec2 ? 2 : 1) + threads - 1) / threads;
+static int layout_chunks(int64_t m, int vec, int threads) {
+    int64_t chunks = (m / vec + threads - 1) / threads;
     return (int)(chunks > 16 ? 16 : (chunks < 1 ? 1 : chunks));
 }
 
-cudaError_t launch_to_tiles(const double* src, int64_t lda, int64_t src_group_stride, double* dst,
-                            const int32_t* cols_dev, int ncols, int64_t dst_col_stride, int nb, int p,
-                            cudaStream_t s) {
+template <class T>
+cudaError_t launch_to_tiles(const T* src, int64_t lda, int64_t src_group_stride, T* dst, const int32_t* cols_dev,
+                            int local_src, int ncols, int64_t dst_col_stride, int nb, int p, int64_t m_valid,
+                            int64_t n_valid, cudaStream_t s) {
     if (ncols <= 0) return cudaSuccess;
-    const int vec2 = ((lda % 2) == 0 && (src_group_stride % 2) == 0 && (((uintptr_t)src) % 16) == 0) ? 1 : 0;
+    constexpr int VEC = 16 / sizeof(T);
+    const bool vec = (lda % VEC) == 0 && (src_group_stride % VEC) == 0 && (m_valid % VEC) == 0 &&
+                     (((uintptr_t)src) % 16) == 0;
     const int threads = 256;
-    dim3 grid(nb * layout_chunks((int64_t)p * nb, vec2, threads), ncols);
-    to_tiles_kernel<<<grid, threads, 0, s>>>(src, lda, src_group_stride, dst, cols_dev, dst_col_stride, nb, p, vec2);
+    dim3 grid(nb * layout_chunks((int64_t)p * nb, vec ? VEC : 1, threads), ncols);
+    if (vec)
+        to_tiles_kernel<T, VEC><<<grid, threads, 0, s>>>(src, lda, src_group_stride, dst, cols_dev, local_src,
+                                                        dst_col_stride, nb, p, m_valid, n_valid);
+    else
+        to_tiles_kernel<T, 1><<<grid, threads, 0, s>>>(src, lda, src_group_stride, dst, cols_dev, local_src,
+                                                      dst_col_stride, nb, p, m_valid, n_valid);
     return cudaGetLastError();
 }
 
-cudaError_t launch_from_tiles(double* dst, int64_t lda, int64_t dst_group_stride, const double* src,
-                              const int32_t* cols_dev, int ncols, int64_t src_col_stride, int nb, int p,
-                              int64_t m_rows, int local_dst, cudaStream_t s) {
-    (void)p;
+template <class T>
+cudaError_t launch_from_tiles(T* dst, int64_t lda, int64_t dst_group_stride, const T* src, const int32_t* cols_dev,
+                              int ncols, int64_t src_col_stride, int nb, int64_t m_rows, int64_t n_valid,
+                              int local_dst, cudaStream_t s) {
     if (ncols <= 0 || m_rows <= 0) return cudaSuccess;
-    const int vec2 = ((lda % 2) == 0 && (dst_group_stride % 2) == 0 && (m_rows % 2) == 0 &&
-                      (((uintptr_t)dst) % 16) == 0) ? 1 : 0;
+    constexpr int VEC = 16 / sizeof(T);
+    const bool vec = (lda % VEC) == 0 && (dst_group_stride % VEC) == 0 && (m_rows % VEC) == 0 &&
+                     (((uintptr_t)dst) % 16) == 0;
     const int threads = 256;
-    dim3 grid(nb * layout_chunks(m_rows, vec2, threads), ncols);
-    from_tiles_kernel<<<grid, threads, 0, s>>>(dst, lda, dst_group_stride, src, cols_dev, src_col_stride, nb,
-                                               m_rows, local_dst, vec2);
+    dim3 grid(nb * layout_chunks(m_rows, vec ? VEC : 1, threads), ncols);
+    if (vec)
+        from_tiles_kernel<T, VEC><<<grid, threads, 0, s>>>(dst, lda, dst_group_stride, src, cols_dev, src_col_stride,
+                                                          nb, m_rows, n_valid, local_dst);
+    else
+        from_tiles_kernel<T, 1><<<grid, threads, 0, s>>>(dst, lda, dst_group_stride, src, cols_dev, src_col_stride,
+                                                        nb, m_rows, n_valid, local_dst);
     return cudaGetLastError();
 }
+template cudaError_t launch_to_tiles<double>(const double*, int64_t, int64_t, double*, const int32_t*, int, int,
+                                             int64_t, int, int, int64_t, int64_t, cudaStream_t);
+template cudaError_t launch_to_tiles<float>(const float*, int64_t, int64_t, float*, const int32_t*, int, int,
+                                            int64_t, int, int, int64_t, int64_t, cudaStream_t);
+template cudaError_t launch_from_tiles<double>(double*, int64_t, int64_t, const double*, const int32_t*, int,
+                                               int64_t, int, int64_t, int64_t, int, cudaStream_t);
+template cudaError_t launch_from_tiles<float>(float*, int64_t, int64_t, const float*, const int32_t*, int,
+                                              int64_t, int, int64_t, int64_t, int, cudaStream_t);
 
 cudaError_t launch_trsv_upper(const double* R, int64_t ldr, double* C, int64_t ldc, int64_t n, int64_t nrhs,
                               cudaStream_t s) {

@@ -234,6 +234,9 @@ tqr_status ensure_io(tqr_plan h, Owner& o) {
     return TQR_OK;
 }
 
+// valid (unpadded) columns of column group j
+int64_t group_cols(const tqr_plan_s* h, int64_t j) { return std::min<int64_t>(h->nb, h->n - j * h->nb); }
+
 tqr_status sync_all(tqr_plan h) {
     for (auto& o : h->owners) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
@@ -293,12 +296,12 @@ static tqr_status validate_guide(int32_t ndev, const int32_t* guide, int32_t gui
 
 tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const int32_t* guide, int32_t guide_len,
                         int32_t rank, int32_t* ops, int64_t cap, int64_t* count) {
-    if (m < 1 || n < 1 || m < n || nb < 1 || n % nb || m % nb || ndev < 1 || rank < 0 || rank >= ndev || !count)
+    if (m < 1 || n < 1 || m < n || nb < 1 || ndev < 1 || rank < 0 || rank >= ndev || !count)
         return fail(nullptr, TQR_ERR_ARG, "schedule: bad arguments");
     std::vector<int32_t> g;
     tqr_status st = validate_guide(ndev, guide, guide_len, g);
     if (st) return st;
-    const int64_t q = n / nb;
+    const int64_t q = (n + nb - 1) / nb;
     std::vector<int32_t> owner_of(q);
     for (int64_t j = 0; j < q; ++j) owner_of[j] = g[j % g.size()];
     std::vector<int32_t> out;
@@ -358,7 +361,6 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     std::vector<int32_t> g;
     tqr_status st = validate_guide(ndev, guide, guide_len, g);
     if (st) return st;
-    if (m % nb || n % nb) return fail(nullptr, TQR_ERR_UNSUPPORTED, "m and n must be multiples of nb in this build");
     if (!supported_nb_ib(nb, ib)) return fail(nullptr, TQR_ERR_UNSUPPORTED, "nb in {64,128,256,512}, ib in {16,32} only");
     if (dtype != TQR_F64) return fail(nullptr, TQR_ERR_UNSUPPORTED, "FP32 path not in this build");
     tqr_options o{};
@@ -377,7 +379,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         return fail(nullptr, TQR_ERR_ARG, "ndev %d > %d visible CUDA devices (set logical_devices)", ndev, ndevices);
 
     tqr_plan h = new tqr_plan_s();
-    h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)(m / nb); h->q = (int)(n / nb);
+    h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)((m + nb - 1) / nb); h->q = (int)((n + nb - 1) / nb);
     h->dtype = dtype; h->ndev = ndev; h->guide = g;
     h->logical = o.logical_devices != 0;
     h->rank = use_nccl ? o.rank : 0;
@@ -528,7 +530,8 @@ tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
         const int nc = (int)o.cols.size();
         if (pi.kind == Mem::Device && pi.dev == o.dev) {
-            CUDA_TRY(h, tqr::launch_to_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, nc, p * tile, (int)nb, (int)p, o.s_upd));
+            CUDA_TRY(h, tqr::launch_to_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, 0, nc, p * tile, (int)nb, (int)p,
+                                             h->m, h->n, o.s_upd));
             h->launches++;
         } else {
             tqr_status st = ensure_io(h, o);
@@ -536,11 +539,12 @@ tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
             for (int lc = 0; lc < nc; ++lc) {
                 const int64_t j = o.cols[lc];
                 CUDA_TRY(h, cudaMemcpy2DAsync(o.io + (int64_t)lc * h->m * nb, h->m * sizeof(double),
-                                              A + j * nb * lda, lda * sizeof(double), h->m * sizeof(double), nb,
-                                              cudaMemcpyDefault, o.s_upd));
+                                              A + j * nb * lda, lda * sizeof(double), h->m * sizeof(double),
+                                              group_cols(h, j), cudaMemcpyDefault, o.s_upd));
             }
-            // io holds the owned columns in local order: group lc at io + lc*m*nb -> use an identity map
-            CUDA_TRY(h, tqr::launch_to_tiles(o.io, h->m, h->m * nb, o.tiles, nullptr, nc, p * tile, (int)nb, (int)p, o.s_upd));
+            // io holds the owned columns in local order: group lc at io + lc*m*nb
+            CUDA_TRY(h, tqr::launch_to_tiles(o.io, h->m, h->m * nb, o.tiles, o.cols_dev, 1, nc, p * tile, (int)nb,
+                                             (int)p, h->m, h->n, o.s_upd));
             h->launches++;
         }
     }
@@ -753,17 +757,18 @@ tqr_status tqr_store_r(tqr_plan h, void* Av, int64_t lda) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
         const int nc = (int)o.cols.size();
         if (pi.kind == Mem::Device && pi.dev == o.dev) {
-            CUDA_TRY(h, tqr::launch_from_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, nc, p * tile, (int)nb, (int)p, h->m, 0, o.s_upd));
+            CUDA_TRY(h, tqr::launch_from_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, nc, p * tile, (int)nb, h->m, h->n, 0, o.s_upd));
             h->launches++;
         } else {
             tqr_status st = ensure_io(h, o);
             if (st) return st;
-            CUDA_TRY(h, tqr::launch_from_tiles(o.io, h->m, h->m * nb, o.tiles, o.cols_dev, nc, p * tile, (int)nb, (int)p, h->m, 1, o.s_upd));
+            CUDA_TRY(h, tqr::launch_from_tiles(o.io, h->m, h->m * nb, o.tiles, o.cols_dev, nc, p * tile, (int)nb, h->m, h->n, 1, o.s_upd));
             h->launches++;
             for (int lc = 0; lc < nc; ++lc) {
                 const int64_t j = o.cols[lc];
                 CUDA_TRY(h, cudaMemcpy2DAsync(A + j * nb * lda, lda * sizeof(double), o.io + (int64_t)lc * h->m * nb,
-                                              h->m * sizeof(double), h->m * sizeof(double), nb, cudaMemcpyDefault, o.s_upd));
+                                              h->m * sizeof(double), h->m * sizeof(double), group_cols(h, j),
+                                              cudaMemcpyDefault, o.s_upd));
             }
         }
     }
@@ -808,7 +813,8 @@ static tqr_status apply_device(tqr_plan h, char trans, double* Bw, int64_t ldw, 
 static tqr_status stage_b(tqr_plan h, const double* B, int64_t ldb, int64_t nrhs, int64_t* nslices, cudaStream_t s) {
     const int64_t pad = (nrhs + 31) / 32 * 32;
     *nslices = pad / 32;
-    const size_t need = (size_t)h->m * pad;
+    const int64_t mp = (int64_t)h->p * h->nb;   // zero-padded rows m..mp-1 (Q = diag(Q_m, I))
+    const size_t need = (size_t)mp * pad;
     if (need > h->bw_elems) {
         if (h->bw) cudaFree(h->bw);
         h->bw = nullptr;
@@ -817,7 +823,7 @@ static tqr_status stage_b(tqr_plan h, const double* B, int64_t ldb, int64_t nrhs
         h->bw_elems = need;
     }
     CUDA_TRY(h, cudaMemsetAsync(h->bw, 0, need * sizeof(double), s));
-    CUDA_TRY(h, cudaMemcpy2DAsync(h->bw, h->m * sizeof(double), B, ldb * sizeof(double), h->m * sizeof(double), nrhs,
+    CUDA_TRY(h, cudaMemcpy2DAsync(h->bw, mp * sizeof(double), B, ldb * sizeof(double), h->m * sizeof(double), nrhs,
                                   cudaMemcpyDefault, s));
     return TQR_OK;
 }
@@ -840,9 +846,10 @@ tqr_status tqr_apply_qt(tqr_plan h, char trans, void* Bv, int64_t ldb, int64_t n
     int64_t nsl = 0;
     st = stage_b(h, B, ldb, nrhs, &nsl, s);
     if (st) return st;
-    st = apply_device(h, trans, h->bw, h->m, nsl, s);
+    const int64_t mp = (int64_t)h->p * h->nb;
+    st = apply_device(h, trans, h->bw, mp, nsl, s);
     if (st) return st;
-    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, h->m * sizeof(double), h->m * sizeof(double), nrhs,
+    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, mp * sizeof(double), h->m * sizeof(double), nrhs,
                                   cudaMemcpyDefault, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     return TQR_OK;
@@ -865,7 +872,8 @@ tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
     int64_t nsl = 0;
     st = stage_b(h, B, ldb, nrhs, &nsl, s);
     if (st) return st;
-    st = apply_device(h, 'T', h->bw, h->m, nsl, s);
+    const int64_t mp = (int64_t)h->p * h->nb;
+    st = apply_device(h, 'T', h->bw, mp, nsl, s);
     if (st) return st;
     // gather R (n x n, column-major) from every owner
     const int64_t n = h->n, nb = h->nb, tile = nb * nb;
@@ -874,7 +882,7 @@ tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
     for (auto& o : h->owners) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, tqr::launch_from_tiles(h->rcm, n, nb * n, o.tiles, o.cols_dev, (int)o.cols.size(), h->p * tile,
-                                           (int)nb, h->p, n, 0, s));
+                                           (int)nb, n, n, 0, s));
         h->launches++;
     }
     const int64_t big = INT64_MAX;
@@ -884,9 +892,9 @@ tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
     CUDA_TRY(h, cudaMemcpyAsync(&first_zero, h->dflag, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     if (first_zero != big) return fail(h, TQR_ERR_SINGULAR, "R(%lld,%lld) == 0", (long long)first_zero, (long long)first_zero);
-    CUDA_TRY(h, tqr::launch_trsv_upper(h->rcm, n, h->bw, h->m, n, nrhs, s));
+    CUDA_TRY(h, tqr::launch_trsv_upper(h->rcm, n, h->bw, mp, n, nrhs, s));
     h->launches++;
-    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, h->m * sizeof(double), n * sizeof(double), nrhs,
+    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, mp * sizeof(double), n * sizeof(double), nrhs,
                                   cudaMemcpyDefault, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     return TQR_OK;

@@ -39,16 +39,19 @@ struct UpdateArgs {
 cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s);
 // nslices CTAs; CTA b works on columns [b*w, b*w + w) counted from group0 (groups are nb wide)
 cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslices, bool trans, cudaStream_t s);
-// src column group of local column lc at src + (cols_dev ? cols[lc] : lc)*src_group_stride (ld = lda)
-// -> tiles at dst + lc*dst_col_stride
-cudaError_t launch_to_tiles(const double* src, int64_t lda, int64_t src_group_stride, double* dst,
-                            const int32_t* cols_dev, int ncols, int64_t dst_col_stride, int nb, int p,
-                            cudaStream_t s);
-// tiles -> column-major rows [0, m_rows) with zeros below the diagonal (global column of local
-// column lc is cols[lc]); destination group at dst + (local_dst ? lc : cols[lc])*dst_group_stride
-cudaError_t launch_from_tiles(double* dst, int64_t lda, int64_t dst_group_stride, const double* src,
-                              const int32_t* cols_dev, int ncols, int64_t src_col_stride, int nb, int p,
-                              int64_t m_rows, int local_dst, cudaStream_t s);
+// a1: src column group of local column lc at src + (local_src ? lc : cols[lc])*src_group_stride
+// (ld = lda) -> tiles at dst + lc*dst_col_stride; rows >= m_valid and global columns >= n_valid -> 0
+template <class T>
+cudaError_t launch_to_tiles(const T* src, int64_t lda, int64_t src_group_stride, T* dst, const int32_t* cols_dev,
+                            int local_src, int ncols, int64_t dst_col_stride, int nb, int p, int64_t m_valid,
+                            int64_t n_valid, cudaStream_t s);
+// a8: tiles -> column-major rows [0, m_rows) of global columns < n_valid, zeros below the diagonal
+// (global column group of local column lc is cols[lc]); destination group at
+// dst + (local_dst ? lc : cols[lc])*dst_group_stride
+template <class T>
+cudaError_t launch_from_tiles(T* dst, int64_t lda, int64_t dst_group_stride, const T* src, const int32_t* cols_dev,
+                              int ncols, int64_t src_col_stride, int nb, int64_t m_rows, int64_t n_valid,
+                              int local_dst, cudaStream_t s);
 cudaError_t launch_trsv_upper(const double* R, int64_t ldr, double* C, int64_t ldc, int64_t n, int64_t nrhs,
                               cudaStream_t s);
 cudaError_t launch_zero_diag_check(const double* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s);

@@ -78,9 +78,16 @@ def test_schedule_covers_dag(L, guide, ndev):
         assert (p - k - 1) * n_up == (p - k - 1) * (q - k - 1)
 
 
+def test_schedule_ragged_sizes(L):
+    """m, n not multiples of nb: zero-padded to whole tiles, q = ceil(n / nb) column tiles."""
+    for (m, n, nb) in [(100, 64, 64), (300, 200, 64), (1000, 777, 256), (65, 65, 64)]:
+        q = -(-n // nb)
+        assert tqr.tqr_schedule(m, n, nb, 1, None, 0) == _expected_schedule(q, [0], 0)
+
+
 def test_schedule_rejects_bad_args(L):
     with pytest.raises(tqr.TqrError):
-        tqr.tqr_schedule(100, 64, 64, 1, None, 0)
+        tqr.tqr_schedule(64, 100, 64, 1, None, 0)      # m < n
     with pytest.raises(tqr.TqrError):
         tqr.tqr_schedule(128, 128, 64, 2, [0, 5], 0)
 

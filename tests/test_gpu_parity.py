@@ -86,6 +86,42 @@ def test_factor_matches_oracle(m, n, nb, ib):
     plan.close()
 
 
+RAGGED = [
+    # (m, n, nb, ib): m and/or n not multiples of nb -> zero-padded tiles
+    (100, 64, 64, 16),      # ragged rows only, 2x1
+    (70, 70, 64, 16),       # 1-element tail column of a square matrix (u = 0 case, reading Q1)
+    (300, 200, 64, 16),     # 5x4 grid, ragged both ways
+    (129, 1, 64, 16),       # single column
+    (1000, 777, 256, 32),   # 4x4 at C2's nb, ragged both ways
+    (1100, 1030, 512, 32),  # 3x3 at nb=512
+    (600, 513, 128, 32),    # last column tile 1 wide
+]
+
+
+@pytest.mark.parametrize("m,n,nb,ib", RAGGED)
+def test_ragged_matches_oracle(m, n, nb, ib):
+    """Ragged tails: R, residual, thin-Q orthogonality, Q^T A top rows and least squares."""
+    A = synthetic.gaussian(m, n, 2000 + m + n + nb)
+    plan, Rg = gpu_qr(A, nb, ib)
+    ref = oracle.qr(A)
+    assert colnorm_rel_err(np.triu(Rg[:n]), ref.R) <= R_TOL
+    assert np.all(np.tril(Rg, -1) == 0.0)
+    Q, res = thin_q_and_residual(plan, A, Rg)
+    assert res <= RES_TOL, res
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0))
+    B = synthetic.gaussian(m, 3, 3000 + m)
+    Bd = dev_colmajor(B)
+    plan.solve_ls(Bd)
+    np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
+    # host-pointer path with lda > m
+    Ah = np.full((m + 3, n), 7.0, order="F")     # rows m.. are outside A: never touched
+    Ah[:m] = A
+    assert tqr.lib().tqr_factor(plan.h, Ah.ctypes.data, m + 3) == 0
+    assert np.array_equal(np.triu(Ah[:n]), np.triu(Rg[:n]))
+    assert np.all(Ah[m:] == 7.0)
+    plan.close()
+
+
 def test_c1_config_full_parity():
     c = synthetic.CONFIGS["C1"]
     A = synthetic.gaussian(c["m"], c["n"], c["seed"])
@@ -216,7 +252,7 @@ def test_integer_and_ill_conditioned_inputs():
 
 def test_errors_and_states():
     with pytest.raises(tqr.TqrError) as e:
-        tqr.Plan(100, 64, 64, 16)           # m not a multiple of nb
+        tqr.Plan(128, 128, 96, 16)          # nb not a built tile size
     assert e.value.status == 7
     with pytest.raises(tqr.TqrError) as e:
         tqr.Plan(64, 128, 64, 16)           # m < n
