@@ -1,7 +1,8 @@
 #!/usr/bin/env python
 """bench.py -- tiled-QR throughput on B200 (BASELINE.json metric).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--dtype f64|f32]
+                    [--impl ours|reference]
 
 metric : tiled QR GFLOP/s = (2mn^2 - 2n^3/3) / t, whole job, plus % of the FP64 tensor peak.
 step   : one pass of the whole hot path over the config's matrix:
@@ -53,6 +54,17 @@ def fp64_peak_tflops():
         return float(d["dmma_tflops"]), d.get("source", "profiles/fp64_peak.json")
     except Exception:
         return 37.2, "nominal 148 SM x 64 FMA/clk x 2 x 1.965 GHz"
+
+
+def fp32_peak_tflops():
+    """FFMA peak (FP32 SIMT pipe): measured by tools/probes/fp32_peak.cu if recorded, else derived
+    from the unit counts: 148 SM x 4 SMSP x 32 lanes x 2 flop x 1.965 GHz = 74.4 TFLOP/s."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "fp32_peak.json")) as f:
+            d = json.load(f)
+        return float(d["ffma_tflops"]), d.get("source", "profiles/fp32_peak.json")
+    except Exception:
+        return 148 * 4 * 32 * 2 * 1.965e-3, "derived: 148 SM x 128 FP32 lanes x 2 x 1.965 GHz"
 
 
 def load_profile_summary(cfg):
@@ -173,6 +185,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default=DEFAULT_CONFIG, choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"],
+                    help="f32: the C5 FP32 configuration (FFMA updates)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-lookahead", action="store_true")
@@ -193,20 +207,23 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
 
     m, n, nb, ib, seed = CONFIGS[args.config]
+    f32 = args.dtype == "f32"
+    tdt = torch.float32 if f32 else torch.float64
+    es = 4 if f32 else 8
     W = max(args.warmup, 3)
     K = max(args.steps, 1)
 
     # ---- inputs (seeded synthetic N(0,1), generated on the device; identical on every rank)
     gen = torch.Generator(device="cuda").manual_seed(seed)
-    A0 = torch.randn((n, m), dtype=torch.float64, device="cuda", generator=gen).t()   # column-major m x n
-    Rout = torch.empty((n, m), dtype=torch.float64, device="cuda").t()
+    A0 = torch.randn((n, m), dtype=tdt, device="cuda", generator=gen).t()   # column-major m x n
+    Rout = torch.empty((n, m), dtype=tdt, device="cuda").t()
 
     nccl_id = None
     if world > 1:
         obj = [tqr.tqr_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
-    plan = tqr.Plan(m, n, nb, ib, ndev=world, rank=rank, world=world, nccl_id=nccl_id,
+    plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, rank=rank, world=world, nccl_id=nccl_id,
                     lookahead=not args.no_lookahead, profile=True)
 
     def step(Ain, Aout):
@@ -250,14 +267,14 @@ def main():
     pcount, pms, pflops = plan.kernel_stats(1, reset=True)
     fl = flops(m, n)
     value = fl / (ms * 1e-3) / 1e9
-    peak, peak_src = fp64_peak_tflops()
+    peak, peak_src = fp32_peak_tflops() if f32 else fp64_peak_tflops()
 
     # ---- e2e: pinned host in, pinned host out, copies inside the timed region
     e2e = None
     if not args.no_e2e:
-        Ah = torch.empty((n, m), dtype=torch.float64, pin_memory=True).t()
+        Ah = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
         Ah.copy_(A0)
-        Rh = torch.empty((n, m), dtype=torch.float64, pin_memory=True).t()
+        Rh = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
         step(Ah, Rh)
         torch.cuda.synchronize()
         barrier()
@@ -272,7 +289,7 @@ def main():
         torch.cuda.synchronize()
         ems = max_over_ranks(e0.elapsed_time(e1) / ke)
         e2e = {"value": round(fl / (ems * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
-               "ms_per_step": round(ems, 3), "h2d_bytes_per_step": 8 * m * n, "d2h_bytes_per_step": 8 * m * n,
+               "ms_per_step": round(ems, 3), "h2d_bytes_per_step": es * m * n, "d2h_bytes_per_step": es * m * n,
                "api": "tqr_load(host) + tqr_factor_tiles + tqr_store_r(host) == tqr_factor on pinned host A"}
         del Ah, Rh
 
@@ -288,19 +305,21 @@ def main():
         # (union of the launches' CUDA-event intervals on the 4 update streams; the launches of
         # one step overlap, so a per-launch average duration would not be a kernel duration)
         achieved = (uflops / (ums * 1e-3) / 1e12) if ucount else None
-        prof = load_profile_summary(args.config)
+        prof = load_profile_summary(args.config + ("_f32" if f32 else ""))
         line = {
             "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak",
             "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
             "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "pct_fp64_peak": round(100.0 * value / 1e3 / (peak * world), 2),
+            "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+            ("pct_fp32_ffma_peak" if f32 else "pct_fp64_peak"): round(100.0 * value / 1e3 / (peak * world), 2),
             "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
-                       "input": "torch.randn N(0,1) fp64 on device (seeded)", "guide": list(range(world)),
+                       "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": list(range(world)),
                        "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
-                       "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (8 * m * n / 2 ** 30)
-                       if 8 * m * n > L2_BYTES else "input fits L2 (no flush)"},
-            "roofline": {"bound": "tensor", "kernel": "update_kernel<512,32,32> (UNMQR+TSMQR chain, DMMA.8x8x4)",
+                       "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (es * m * n / 2 ** 30)
+                       if es * m * n > L2_BYTES else "input fits L2 (no flush)"},
+            "roofline": {"bound": "alu" if f32 else "tensor",
+                         "kernel": "update_kernel32<512,32,32> (UNMQR+TSMQR chain, FFMA)" if f32 else
+                         "update_kernel<512,32,32> (UNMQR+TSMQR chain, DMMA.8x8x4)",
                          "achieved": round(achieved, 3) if achieved else None, "peak": peak, "unit": "TFLOP/s",
                          "frac": round(achieved / peak, 4) if achieved else None,
                          "traffic": prof.get("dram_bytes_per_launch"),

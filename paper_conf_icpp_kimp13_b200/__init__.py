@@ -8,7 +8,8 @@ factorisation runs in the CUDA kernels of ``csrc/``.  There is no CPU fallback: 
 library cannot be loaded, every call raises.
 
 Arrays: torch tensors (CUDA or CPU) or numpy arrays, column-major (stride(0) == 1 for torch,
-Fortran order for numpy), dtype float64.  The leading dimension is taken from the array.
+Fortran order for numpy), dtype float64 (TQR_F64 plans) or float32 (TQR_F32 plans).  The leading
+dimension is taken from the array.
 """
 from __future__ import annotations
 
@@ -93,13 +94,20 @@ def _i32_array(vals):
     return arr, len(vals)
 
 
-def _ptr_ld(x, rows: int):
-    """(pointer, leading dimension) of a column-major 2-D torch tensor or numpy array."""
+_PLAN_DTYPE = {}   # plan handle value -> TQR_F64 / TQR_F32 (argument checking only)
+
+
+def _ptr_ld(x, rows: int, h=None):
+    """(pointer, leading dimension) of a column-major 2-D torch tensor or numpy array whose element
+    type matches the plan's dtype."""
+    want = _PLAN_DTYPE.get(getattr(h, "value", None), None)
     try:
         import torch
         if isinstance(x, torch.Tensor):
-            if x.dtype != torch.float64:
-                raise TypeError("tensor must be float64")
+            tt = {torch.float64: TQR_F64, torch.float32: TQR_F32}.get(x.dtype)
+            if tt is None or (want is not None and tt != want):
+                raise TypeError("tensor dtype %s does not match the plan (float64 for TQR_F64, float32 for TQR_F32)"
+                                % x.dtype)
             if x.dim() == 1:
                 return x.data_ptr(), max(rows, x.shape[0])
             if x.stride(0) != 1:
@@ -109,8 +117,9 @@ def _ptr_ld(x, rows: int):
         pass
     import numpy as np
     if isinstance(x, np.ndarray):
-        if x.dtype != np.float64:
-            raise TypeError("array must be float64")
+        tt = {np.dtype(np.float64): TQR_F64, np.dtype(np.float32): TQR_F32}.get(x.dtype)
+        if tt is None or (want is not None and tt != want):
+            raise TypeError("array dtype %s does not match the plan" % x.dtype)
         if x.ndim == 1:
             return x.ctypes.data, max(rows, x.shape[0])
         if not x.flags.f_contiguous:
@@ -132,16 +141,17 @@ def tqr_create(m, n, nb, ib, dtype=TQR_F64, ndev=1, guide=None, logical_devices=
     st = lib().tqr_create_ex(int(m), int(n), int(nb), int(ib), int(dtype), int(ndev), g, glen, ctypes.byref(opt),
                              ctypes.byref(h))
     _check(st, None)
+    _PLAN_DTYPE[h.value] = int(dtype)
     return h
 
 
 def tqr_factor(h, A):
-    ptr, ld = _ptr_ld(A, 0)
+    ptr, ld = _ptr_ld(A, 0, h)
     _check(lib().tqr_factor(h, ptr, ld), h)
 
 
 def tqr_load(h, A):
-    ptr, ld = _ptr_ld(A, 0)
+    ptr, ld = _ptr_ld(A, 0, h)
     _check(lib().tqr_load(h, ptr, ld), h)
 
 
@@ -150,24 +160,25 @@ def tqr_factor_tiles(h):
 
 
 def tqr_store_r(h, A):
-    ptr, ld = _ptr_ld(A, 0)
+    ptr, ld = _ptr_ld(A, 0, h)
     _check(lib().tqr_store_r(h, ptr, ld), h)
 
 
 def tqr_apply_qt(h, B, trans="T"):
-    ptr, ld = _ptr_ld(B, B.shape[0])
+    ptr, ld = _ptr_ld(B, B.shape[0], h)
     nrhs = 1 if len(B.shape) == 1 else B.shape[1]
     _check(lib().tqr_apply_qt(h, trans.encode()[:1], ptr, ld, nrhs), h)
 
 
 def tqr_solve_ls(h, B):
-    ptr, ld = _ptr_ld(B, B.shape[0])
+    ptr, ld = _ptr_ld(B, B.shape[0], h)
     nrhs = 1 if len(B.shape) == 1 else B.shape[1]
     _check(lib().tqr_solve_ls(h, ptr, ld, nrhs), h)
 
 
 def tqr_destroy(h):
     if h:
+        _PLAN_DTYPE.pop(h.value, None)
         lib().tqr_destroy(h)
 
 

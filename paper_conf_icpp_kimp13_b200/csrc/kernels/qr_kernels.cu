@@ -286,27 +286,27 @@ __global__ void from_tiles_kernel(T* __restrict__ dst, int64_t lda, int64_t dst_
     }
 }
 
-// Back substitution R X = C for the n x n upper-triangular R held in tile layout (panel
-// column owner storage gathered into `Rcm`, column-major n x n, ld = ldr).  One CTA per
-// right-hand side; columns of R are streamed (Eq. 3).
-__global__ void trsv_upper_kernel(const double* __restrict__ R, int64_t ldr, double* __restrict__ C,
-                                  int64_t ldc, int64_t n) {
-    double* x = C + (int64_t)blockIdx.x * ldc;
-    __shared__ double xi_s;
+// Back substitution R X = C for the n x n upper-triangular R (gathered column-major into R,
+// ld = ldr).  One CTA per right-hand side; columns of R are streamed (Eq. 3).
+template <class T>
+__global__ void trsv_upper_kernel(const T* __restrict__ R, int64_t ldr, T* __restrict__ C, int64_t ldc, int64_t n) {
+    T* x = C + (int64_t)blockIdx.x * ldc;
+    __shared__ T xi_s;
     for (int64_t i = n - 1; i >= 0; --i) {
         if (threadIdx.x == 0) xi_s = x[i] / R[i + i * ldr];
         __syncthreads();
-        const double xi = xi_s;
-        const double* rc = R + i * ldr;
+        const T xi = xi_s;
+        const T* rc = R + i * ldr;
         for (int64_t r = threadIdx.x; r < i; r += blockDim.x) x[r] -= rc[r] * xi;
         if (threadIdx.x == 0) x[i] = xi;
         __syncthreads();
     }
 }
 
-__global__ void zero_diag_check_kernel(const double* __restrict__ R, int64_t ldr, int64_t n, int64_t* first_zero) {
+template <class T>
+__global__ void zero_diag_check_kernel(const T* __restrict__ R, int64_t ldr, int64_t n, int64_t* first_zero) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        if (R[i + i * ldr] == 0.0) atomicMin(reinterpret_cast<unsigned long long*>(first_zero), (unsigned long long)i);
+        if (R[i + i * ldr] == T(0)) atomicMin(reinterpret_cast<unsigned long long*>(first_zero), (unsigned long long)i);
 }
 
 // ============================================================================ launchers
@@ -435,17 +435,22 @@ template cudaError_t launch_from_tiles<double>(double*, int64_t, int64_t, const 
 template cudaError_t launch_from_tiles<float>(float*, int64_t, int64_t, const float*, const int32_t*, int,
                                               int64_t, int, int64_t, int64_t, int, cudaStream_t);
 
-cudaError_t launch_trsv_upper(const double* R, int64_t ldr, double* C, int64_t ldc, int64_t n, int64_t nrhs,
-                              cudaStream_t s) {
+template <class T>
+cudaError_t launch_trsv_upper(const T* R, int64_t ldr, T* C, int64_t ldc, int64_t n, int64_t nrhs, cudaStream_t s) {
     if (nrhs <= 0) return cudaSuccess;
-    trsv_upper_kernel<<<(unsigned)nrhs, 256, 0, s>>>(R, ldr, C, ldc, n);
+    trsv_upper_kernel<T><<<(unsigned)nrhs, 256, 0, s>>>(R, ldr, C, ldc, n);
     return cudaGetLastError();
 }
 
-cudaError_t launch_zero_diag_check(const double* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s) {
-    zero_diag_check_kernel<<<64, 256, 0, s>>>(R, ldr, n, first_zero);
+template <class T>
+cudaError_t launch_zero_diag_check(const T* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s) {
+    zero_diag_check_kernel<T><<<64, 256, 0, s>>>(R, ldr, n, first_zero);
     return cudaGetLastError();
 }
+template cudaError_t launch_trsv_upper<double>(const double*, int64_t, double*, int64_t, int64_t, int64_t, cudaStream_t);
+template cudaError_t launch_trsv_upper<float>(const float*, int64_t, float*, int64_t, int64_t, int64_t, cudaStream_t);
+template cudaError_t launch_zero_diag_check<double>(const double*, int64_t, int64_t, int64_t*, cudaStream_t);
+template cudaError_t launch_zero_diag_check<float>(const float*, int64_t, int64_t, int64_t*, cudaStream_t);
 
 size_t panel_smem_bytes(int nb, int ib) {
 #define TQR_PS(NB_, IB_) if (nb == NB_ && ib == IB_) return sizeof(Smem<NB_, IB_, IB_, true>);

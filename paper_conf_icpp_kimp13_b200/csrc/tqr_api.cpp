@@ -44,15 +44,21 @@ struct Owner {
     std::vector<int32_t> cols;      // global column tiles owned (ascending)
     std::vector<int32_t> lidx;      // global j -> local index or -1
     int32_t* cols_dev = nullptr;
-    double* tiles = nullptr;        // ncols * p * nb*nb
-    double* T = nullptr;            // ncols * p * ib*nb
-    double* Vimg = nullptr;         // ncols * p * nb*nb  stage images of the reflector tiles (update-kernel operand)
-    double* Vexp = nullptr;         // ncols * nb*nb      stage image of the explicit V of each diagonal tile
-    double* rb_tiles[2] = {nullptr, nullptr};
-    double* rb_T[2] = {nullptr, nullptr};
-    double* rb_V[2] = {nullptr, nullptr};
+    // element type = the plan's dtype (double or float); sizes in elements
+    void* tiles = nullptr;          // ncols * p * nb*nb
+    void* T = nullptr;              // ncols * p * ib*nb
+    void* Vimg = nullptr;           // ncols * p * vt     stage images of the reflector tiles (update-kernel operand)
+    void* Vexp = nullptr;           // ncols * vt         stage image of the explicit V of each diagonal tile
+    void* rb_tiles[2] = {nullptr, nullptr};
+    void* rb_T[2] = {nullptr, nullptr};
+    void* rb_V[2] = {nullptr, nullptr};
     unsigned* flags = nullptr;      // p * (nb/ib)
-    double* io = nullptr;           // m x (nb*ncols) column-major mirror for host / remote I/O
+    void* io = nullptr;             // m x (nb*ncols) column-major mirror for host / remote I/O
+    // FP32 plans: FP64 scratch of one panel column (the panel is factored in FP64, then narrowed)
+    double* sc_col = nullptr;       // p * nb*nb
+    double* sc_T = nullptr;         // p * ib*nb
+    double* sc_Vimg = nullptr;      // p * nb*nb
+    double* sc_Vexp = nullptr;      // nb*nb
     cudaStream_t s_panel = nullptr, s_upd = nullptr, s_comm = nullptr;
     std::vector<cudaStream_t> s_u;                  // bulk-update streams (column lc -> s_u[lc % S])
     std::vector<cudaEvent_t> ev_panel, ev_recv, ev_look;
@@ -74,6 +80,8 @@ struct tqr_plan_s {
     int64_t m = 0, n = 0;
     int nb = 0, ib = 0, p = 0, q = 0;
     tqr_dtype dtype = TQR_F64;
+    int es = 8;                     // element size in bytes
+    int64_t vt = 0;                 // elements of one reflector-tile stage image (F64: nb*nb)
     int ndev = 1;
     std::vector<int32_t> guide;
     std::vector<int32_t> owner_of;  // size q
@@ -91,13 +99,17 @@ struct tqr_plan_s {
     KStat stats[4];
     int64_t launches = 0;
     // apply / solve workspace (single-device plans)
-    double* bw = nullptr;
+    void* bw = nullptr;
     size_t bw_elems = 0;
-    double* rcm = nullptr;
+    void* rcm = nullptr;
     int64_t* dflag = nullptr;
 
     bool nccl_mode = false;         // one process per GPU, panels broadcast with NCCL
     bool multiproc() const { return nccl_mode; }
+    bool f32() const { return dtype == TQR_F32; }
+    // p + e elements
+    template <class E = void>
+    E* at(void* ptr, int64_t e) const { return reinterpret_cast<E*>(static_cast<char*>(ptr) + e * es); }
     Owner* local(int d) {
         if (multiproc()) return (d == rank) ? &owners[0] : nullptr;
         return &owners[d];
@@ -158,6 +170,7 @@ void free_owner(Owner& o) {
     cudaSetDevice(o.dev);
     auto F = [](void* p) { if (p) cudaFree(p); };
     F(o.cols_dev); F(o.tiles); F(o.Vimg); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
+    F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp);
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
     for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref})
         for (auto e : *v) if (e) cudaEventDestroy(e);
@@ -230,7 +243,7 @@ tqr_status sync_entry(tqr_plan h, const PtrInfo& pi) {
 tqr_status ensure_io(tqr_plan h, Owner& o) {
     if (o.io || o.cols.empty()) return TQR_OK;
     CUDA_TRY(h, cudaSetDevice(o.dev));
-    CUDA_TRY(h, cudaMalloc(&o.io, sizeof(double) * (size_t)h->m * h->nb * o.cols.size()));
+    CUDA_TRY(h, cudaMalloc(&o.io, (size_t)h->es * h->m * h->nb * o.cols.size()));
     return TQR_OK;
 }
 
@@ -362,7 +375,6 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     tqr_status st = validate_guide(ndev, guide, guide_len, g);
     if (st) return st;
     if (!supported_nb_ib(nb, ib)) return fail(nullptr, TQR_ERR_UNSUPPORTED, "nb in {64,128,256,512}, ib in {16,32} only");
-    if (dtype != TQR_F64) return fail(nullptr, TQR_ERR_UNSUPPORTED, "FP32 path not in this build");
     tqr_options o{};
     if (opt) o = *opt;
     // NCCL mode: world > 1, or a single-rank communicator when an nccl_id is given explicitly
@@ -381,6 +393,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     tqr_plan h = new tqr_plan_s();
     h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)((m + nb - 1) / nb); h->q = (int)((n + nb - 1) / nb);
     h->dtype = dtype; h->ndev = ndev; h->guide = g;
+    h->es = (dtype == TQR_F32) ? 4 : 8;
+    h->vt = (dtype == TQR_F32) ? tqr::f32_img_tile(nb, ib) : (int64_t)nb * nb;
     h->logical = o.logical_devices != 0;
     h->rank = use_nccl ? o.rank : 0;
     h->world = world;
@@ -438,17 +452,23 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         }
         if (!ok) return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
         const size_t nc = ow.cols.size();
-        auto alloc = [&](double** ptr, size_t elems) -> bool {
-            if (elems == 0) return true;
-            if (cudaMalloc(ptr, elems * sizeof(double)) != cudaSuccess) { cudaGetLastError(); return false; }
+        const int64_t vt = h->vt;
+        auto allocb = [&](void** ptr, size_t bytes) -> bool {
+            if (bytes == 0) return true;
+            if (cudaMalloc(ptr, bytes) != cudaSuccess) { cudaGetLastError(); return false; }
+            if (cudaMemset(*ptr, 0, bytes) != cudaSuccess) { cudaGetLastError(); return false; }
             return true;
         };
-        if (!alloc(&ow.tiles, nc * p * tile) || !alloc(&ow.Vimg, nc * p * tile) || !alloc(&ow.T, nc * p * tsz) ||
-            !alloc(&ow.Vexp, nc * tile))
+        auto alloc = [&](void** ptr, size_t elems) -> bool { return allocb(ptr, elems * h->es); };
+        auto alloc64 = [&](double** ptr, size_t elems) -> bool { return allocb((void**)ptr, elems * sizeof(double)); };
+        if (!alloc(&ow.tiles, nc * p * tile) || !alloc(&ow.Vimg, nc * p * vt) || !alloc(&ow.T, nc * p * tsz) ||
+            !alloc(&ow.Vexp, nc * vt))
             return bail(fail(h, TQR_ERR_ALLOC, "tile storage allocation failed"));
+        if (nc && h->f32() &&
+            (!alloc64(&ow.sc_col, p * tile) || !alloc64(&ow.sc_T, p * tsz) || !alloc64(&ow.sc_Vimg, p * tile) ||
+             !alloc64(&ow.sc_Vexp, tile)))
+            return bail(fail(h, TQR_ERR_ALLOC, "FP64 panel scratch allocation failed"));
         if (nc) {
-            if (cudaMemset(ow.T, 0, nc * p * tsz * sizeof(double)) != cudaSuccess)
-                return bail(fail(h, TQR_ERR_CUDA, "memset"));
             if (cudaMalloc(&ow.cols_dev, nc * sizeof(int32_t)) != cudaSuccess ||
                 cudaMemcpy(ow.cols_dev, ow.cols.data(), nc * sizeof(int32_t), cudaMemcpyHostToDevice) != cudaSuccess)
                 return bail(fail(h, TQR_ERR_ALLOC, "cols allocation failed"));
@@ -460,7 +480,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
                 for (int j = k + 1; j < h->q; ++j) if (h->owner_of[j] == ow.id) { need_rb = true; break; }
         if (need_rb)
             for (int s = 0; s < 2; ++s)
-                if (!alloc(&ow.rb_tiles[s], p * tile) || !alloc(&ow.rb_T[s], p * tsz) || !alloc(&ow.rb_V[s], tile))
+                if (!alloc(&ow.rb_tiles[s], p * vt) || !alloc(&ow.rb_T[s], p * tsz) || !alloc(&ow.rb_V[s], vt))
                     return bail(fail(h, TQR_ERR_ALLOC, "receive buffer allocation failed"));
         if (nc) {
             const size_t nfl = (size_t)p * (nb / ib) * 5;   // F + up to 4 sub-slice flags
@@ -515,14 +535,60 @@ tqr_status tqr_kernel_stats(tqr_plan h, int32_t which, int64_t* count, double* m
     return TQR_OK;
 }
 
+// ------------------------------------------------------------------ typed launch helpers
+namespace {
+cudaError_t to_tiles(const tqr_plan_s* h, const void* src, int64_t lda, int64_t gstride, void* dst, const int32_t* cols,
+                     int local_src, int nc, cudaStream_t s) {
+    const int64_t colsz = (int64_t)h->p * h->nb * h->nb;
+    if (h->f32())
+        return tqr::launch_to_tiles<float>((const float*)src, lda, gstride, (float*)dst, cols, local_src, nc, colsz,
+                                           h->nb, h->p, h->m, h->n, s);
+    return tqr::launch_to_tiles<double>((const double*)src, lda, gstride, (double*)dst, cols, local_src, nc, colsz,
+                                        h->nb, h->p, h->m, h->n, s);
+}
+cudaError_t from_tiles(const tqr_plan_s* h, void* dst, int64_t lda, int64_t gstride, const void* src,
+                       const int32_t* cols, int nc, int64_t m_rows, int64_t n_valid, int local_dst, cudaStream_t s) {
+    const int64_t colsz = (int64_t)h->p * h->nb * h->nb;
+    if (h->f32())
+        return tqr::launch_from_tiles<float>((float*)dst, lda, gstride, (const float*)src, cols, nc, colsz, h->nb,
+                                             m_rows, n_valid, local_dst, s);
+    return tqr::launch_from_tiles<double>((double*)dst, lda, gstride, (const double*)src, cols, nc, colsz, h->nb,
+                                          m_rows, n_valid, local_dst, s);
+}
+// Reflector data of panel k as seen by an update: images V (tile i at V + i*vt), T, explicit V.
+struct PanelRefs {
+    void* V;
+    void* T;
+    void* Vexp;
+};
+cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col_stride, int64_t tile_stride,
+                   int64_t ld, int group0, int gstride, int k, int w, int nslices, bool trans, cudaStream_t s) {
+    if (h->f32()) {
+        tqr::UpdateArgsT<float> u;
+        u.V = (const float*)r.V; u.T = (const float*)r.T; u.Vexp = (const float*)r.Vexp; u.X = (float*)X;
+        u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
+        u.group0 = group0; u.gstride = gstride; u.k = k; u.p = h->p; u.do_unmqr = 1;
+        return tqr::launch_update_f32(h->nb, h->ib, w, u, nslices, trans, s);
+    }
+    tqr::UpdateArgs u;
+    u.V = (const double*)r.V; u.T = (const double*)r.T; u.Vexp = (const double*)r.Vexp; u.X = (double*)X;
+    u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
+    u.group0 = group0; u.gstride = gstride; u.k = k; u.p = h->p; u.do_unmqr = 1;
+    return tqr::launch_update(h->nb, h->ib, w, u, nslices, trans, s);
+}
+PanelRefs own_refs(const tqr_plan_s* h, Owner& O, int lc) {
+    const int64_t p = h->p, tsz = (int64_t)h->ib * h->nb;
+    return {h->at(O.Vimg, lc * p * h->vt), h->at(O.T, lc * p * tsz), h->at(O.Vexp, lc * h->vt)};
+}
+}  // namespace
+
 // ------------------------------------------------------------------ a1: load
-tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
+tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
-    if (!Av || lda < h->m) return fail(h, TQR_ERR_ARG, "load: A is NULL or lda < m");
-    const double* A = static_cast<const double*>(Av);
+    if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "load: A is NULL or lda < m");
     const PtrInfo pi = classify(A);
-    const int64_t p = h->p, nb = h->nb, tile = nb * nb;
+    const int64_t nb = h->nb, es = h->es;
     h->factored = false;
     { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
     for (auto& o : h->owners) {
@@ -530,21 +596,19 @@ tqr_status tqr_load(tqr_plan h, const void* Av, int64_t lda) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
         const int nc = (int)o.cols.size();
         if (pi.kind == Mem::Device && pi.dev == o.dev) {
-            CUDA_TRY(h, tqr::launch_to_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, 0, nc, p * tile, (int)nb, (int)p,
-                                             h->m, h->n, o.s_upd));
+            CUDA_TRY(h, to_tiles(h, A, lda, nb * lda, o.tiles, o.cols_dev, 0, nc, o.s_upd));
             h->launches++;
         } else {
             tqr_status st = ensure_io(h, o);
             if (st) return st;
             for (int lc = 0; lc < nc; ++lc) {
                 const int64_t j = o.cols[lc];
-                CUDA_TRY(h, cudaMemcpy2DAsync(o.io + (int64_t)lc * h->m * nb, h->m * sizeof(double),
-                                              A + j * nb * lda, lda * sizeof(double), h->m * sizeof(double),
+                CUDA_TRY(h, cudaMemcpy2DAsync(h->at(o.io, (int64_t)lc * h->m * nb), h->m * es,
+                                              static_cast<const char*>(A) + j * nb * lda * es, lda * es, h->m * es,
                                               group_cols(h, j), cudaMemcpyDefault, o.s_upd));
             }
             // io holds the owned columns in local order: group lc at io + lc*m*nb
-            CUDA_TRY(h, tqr::launch_to_tiles(o.io, h->m, h->m * nb, o.tiles, o.cols_dev, 1, nc, p * tile, (int)nb,
-                                             (int)p, h->m, h->n, o.s_upd));
+            CUDA_TRY(h, to_tiles(h, o.io, h->m, h->m * nb, o.tiles, o.cols_dev, 1, nc, o.s_upd));
             h->launches++;
         }
     }
@@ -564,13 +628,45 @@ double union_ms(std::vector<std::pair<double, double>>& iv) {
     if (ce > cs) tot += ce - cs;
     return tot;
 }
+
+// PANEL(k) on its owner's panel stream.  FP64: the panel kernel factors the owner's tiles in
+// place.  FP32: widen tiles k..p-1 of the column into the FP64 scratch column, factor there,
+// narrow R / reflectors / T / stage images back (qr_kernels_f32.cu).
+tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
+    const int p = h->p, nb = h->nb, ib = h->ib;
+    const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile;
+    const int lc = O.lidx[k];
+    tqr::PanelArgs a;
+    a.flags = O.flags;
+    a.epoch = epoch;
+    a.k = k;
+    a.p = p;
+    if (!h->f32()) {
+        a.col = h->at<double>(O.tiles, lc * colsz);
+        a.Vimg = h->at<double>(O.Vimg, lc * colsz);
+        a.T = h->at<double>(O.T, lc * (int64_t)p * tsz);
+        a.Vexp = h->at<double>(O.Vexp, lc * tile);
+        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O.s_panel));
+        h->launches++;
+        return TQR_OK;
+    }
+    CUDA_TRY(h, tqr::launch_widen(h->at<float>(O.tiles, lc * colsz + k * tile), O.sc_col + k * tile,
+                                  (int64_t)(p - k) * tile, O.s_panel));
+    a.col = O.sc_col; a.Vimg = O.sc_Vimg; a.T = O.sc_T; a.Vexp = O.sc_Vexp;
+    CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O.s_panel));
+    const PanelRefs r = own_refs(h, O, lc);
+    CUDA_TRY(h, tqr::launch_narrow_panel(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz), (float*)r.T,
+                                         (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
+    h->launches += 3;
+    return TQR_OK;
+}
 }  // namespace
 
 tqr_status tqr_factor_tiles(tqr_plan h) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     const int p = h->p, q = h->q, nb = h->nb, ib = h->ib, S = h->nstreams;
-    const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile;
+    const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile, vt = h->vt;
     const unsigned epoch0 = h->epoch;
     h->epoch += (unsigned)q + 1;
     // order all owner streams after whatever ran before (load, previous calls)
@@ -594,23 +690,13 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
         if (O) {
             CUDA_TRY(h, cudaSetDevice(O->dev));
             if (k > 0 && !h->lookahead) { tqr_status st = wait_all_u(*O, O->s_panel, k - 1); if (st) return st; }
-            const int lc = O->lidx[k];
-            PanelArgs a;
-            a.col = O->tiles + lc * colsz;
-            a.Vimg = O->Vimg + lc * colsz;
-            a.T = O->T + lc * (int64_t)p * tsz;
-            a.Vexp = O->Vexp + lc * tile;
-            a.flags = O->flags;
-            a.epoch = epoch0 + (unsigned)k + 1;
-            a.k = k;
-            a.p = p;
             if (h->profile) CUDA_TRY(h, cudaEventRecord(O->tp0[k], O->s_panel));
-            CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O->s_panel));
-            h->launches++;
+            tqr_status st = launch_panel_step(h, *O, k, epoch0 + (unsigned)k + 1);
+            if (st) return st;
             if (h->profile) { CUDA_TRY(h, cudaEventRecord(O->tp1[k], O->s_panel)); O->tp_used[k] = 1; }
             CUDA_TRY(h, cudaEventRecord(O->ev_panel[k], O->s_panel));
         }
-        // ---- BCAST(k): the reflector tiles k..p-1, their T factors and the explicit V
+        // ---- BCAST(k): the reflector-tile images k..p-1, their T factors and the explicit V
         if (h->multiproc()) {
             Owner& R = h->owners[0];
             CUDA_TRY(h, cudaSetDevice(R.dev));
@@ -622,17 +708,14 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 if (st) return st;
                 CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
             }
-            double *bt, *bT, *bV;
-            if (root) {
-                const int lc = R.lidx[k];
-                bt = R.Vimg + lc * colsz; bT = R.T + lc * (int64_t)p * tsz; bV = R.Vexp + lc * tile;
-            } else {
-                bt = R.rb_tiles[slot]; bT = R.rb_T[slot]; bV = R.rb_V[slot];
-            }
+            PanelRefs b = root ? own_refs(h, R, R.lidx[k]) : PanelRefs{R.rb_tiles[slot], R.rb_T[slot], R.rb_V[slot]};
+            const ncclDataType_t dt = h->f32() ? ncclFloat32 : ncclFloat64;
+            void* bv = h->at(b.V, k * vt);
+            void* bt = h->at(b.T, k * tsz);
             NCCL_TRY(h, h->nccl->GroupStart());
-            NCCL_TRY(h, h->nccl->Broadcast(bt + k * tile, bt + k * tile, (size_t)(p - k) * tile, ncclFloat64, ok, h->comm, R.s_comm));
-            NCCL_TRY(h, h->nccl->Broadcast(bT + k * tsz, bT + k * tsz, (size_t)(p - k) * tsz, ncclFloat64, ok, h->comm, R.s_comm));
-            NCCL_TRY(h, h->nccl->Broadcast(bV, bV, (size_t)tile, ncclFloat64, ok, h->comm, R.s_comm));
+            NCCL_TRY(h, h->nccl->Broadcast(bv, bv, (size_t)(p - k) * vt, dt, ok, h->comm, R.s_comm));
+            NCCL_TRY(h, h->nccl->Broadcast(bt, bt, (size_t)(p - k) * tsz, dt, ok, h->comm, R.s_comm));
+            NCCL_TRY(h, h->nccl->Broadcast(b.Vexp, b.Vexp, (size_t)vt, dt, ok, h->comm, R.s_comm));
             NCCL_TRY(h, h->nccl->GroupEnd());
             CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
         } else {
@@ -649,13 +732,13 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     if (st) return st;
                     CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_look[k - 2], 0));
                 }
-                const int lc = O->lidx[k];
-                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_tiles[slot] + k * tile, D.dev, O->Vimg + lc * colsz + k * tile,
-                                                O->dev, sizeof(double) * (size_t)(p - k) * tile, D.s_comm));
-                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_T[slot] + k * tsz, D.dev, O->T + lc * (int64_t)p * tsz + k * tsz,
-                                                O->dev, sizeof(double) * (size_t)(p - k) * tsz, D.s_comm));
-                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, O->Vexp + lc * tile, O->dev,
-                                                sizeof(double) * (size_t)tile, D.s_comm));
+                const PanelRefs src = own_refs(h, *O, O->lidx[k]);
+                const size_t es = h->es;
+                CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_tiles[slot], k * vt), D.dev, h->at(src.V, k * vt), O->dev,
+                                                es * (size_t)(p - k) * vt, D.s_comm));
+                CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_T[slot], k * tsz), D.dev, h->at(src.T, k * tsz), O->dev,
+                                                es * (size_t)(p - k) * tsz, D.s_comm));
+                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, src.Vexp, O->dev, es * (size_t)vt, D.s_comm));
                 CUDA_TRY(h, cudaEventRecord(D.ev_recv[k], D.s_comm));
             }
         }
@@ -663,16 +746,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
         for (auto& D : h->owners) {
             CUDA_TRY(h, cudaSetDevice(D.dev));
             const bool mine = (D.id == ok);
-            UpdateArgs u;
-            if (mine) {
-                const int lc = D.lidx[k];
-                u.V = D.Vimg + lc * colsz; u.T = D.T + lc * (int64_t)p * tsz; u.Vexp = D.Vexp + lc * tile;
-            } else {
-                const int slot = k & 1;
-                u.V = D.rb_tiles[slot]; u.T = D.rb_T[slot]; u.Vexp = D.rb_V[slot];
-            }
-            u.X = D.tiles; u.col_stride = colsz; u.tile_stride = tile; u.ld = nb;
-            u.k = k; u.p = p; u.do_unmqr = 1; u.gstride = 1;
+            const int slot = k & 1;
+            const PanelRefs r = mine ? own_refs(h, D, D.lidx[k]) : PanelRefs{D.rb_tiles[slot], D.rb_T[slot], D.rb_V[slot]};
             cudaEvent_t ready = mine ? D.ev_panel[k] : D.ev_recv[k];
             // local columns j > k form a suffix [first, ncols) of D.cols
             int first = (int)(std::upper_bound(D.cols.begin(), D.cols.end(), k) - D.cols.begin());
@@ -682,8 +757,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 // lookahead: column k+1 first, on the high-priority panel stream
                 CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, ready, 0));
                 if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_u[first % S][k - 1], 0));
-                u.group0 = first;
-                CUDA_TRY(h, tqr::launch_update(nb, ib, w_look(h), u, nb / w_look(h), true, D.s_panel));
+                const int wl = w_look(h);
+                CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, D.s_panel));
                 h->launches++;
                 first += 1;
             }
@@ -696,10 +771,9 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 cudaStream_t su = D.s_u[uu];
                 if (ng > 0) {
                     CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
-                    u.group0 = g0;
-                    u.gstride = S;
                     if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[uu][k], su));
-                    CUDA_TRY(h, tqr::launch_update(nb, ib, w_bulk(h), u, ng * (nb / w_bulk(h)), true, su));
+                    const int wb = w_bulk(h);
+                    CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, S, k, wb, ng * (nb / wb), true, su));
                     h->launches++;
                     if (h->profile) {
                         CUDA_TRY(h, cudaEventRecord(D.tm1[uu][k], su));
@@ -743,32 +817,31 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
 }
 
 // ------------------------------------------------------------------ a8: R out
-tqr_status tqr_store_r(tqr_plan h, void* Av, int64_t lda) {
+tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "store_r before factor");
-    if (!Av || lda < h->m) return fail(h, TQR_ERR_ARG, "store_r: A is NULL or lda < m");
-    double* A = static_cast<double*>(Av);
+    if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "store_r: A is NULL or lda < m");
     const PtrInfo pi = classify(A);
-    const int64_t p = h->p, nb = h->nb, tile = nb * nb;
+    const int64_t nb = h->nb, es = h->es;
     { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
     for (auto& o : h->owners) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, cudaSetDevice(o.dev));
         const int nc = (int)o.cols.size();
         if (pi.kind == Mem::Device && pi.dev == o.dev) {
-            CUDA_TRY(h, tqr::launch_from_tiles(A, lda, nb * lda, o.tiles, o.cols_dev, nc, p * tile, (int)nb, h->m, h->n, 0, o.s_upd));
+            CUDA_TRY(h, from_tiles(h, A, lda, nb * lda, o.tiles, o.cols_dev, nc, h->m, h->n, 0, o.s_upd));
             h->launches++;
         } else {
             tqr_status st = ensure_io(h, o);
             if (st) return st;
-            CUDA_TRY(h, tqr::launch_from_tiles(o.io, h->m, h->m * nb, o.tiles, o.cols_dev, nc, p * tile, (int)nb, h->m, h->n, 1, o.s_upd));
+            CUDA_TRY(h, from_tiles(h, o.io, h->m, h->m * nb, o.tiles, o.cols_dev, nc, h->m, h->n, 1, o.s_upd));
             h->launches++;
             for (int lc = 0; lc < nc; ++lc) {
                 const int64_t j = o.cols[lc];
-                CUDA_TRY(h, cudaMemcpy2DAsync(A + j * nb * lda, lda * sizeof(double), o.io + (int64_t)lc * h->m * nb,
-                                              h->m * sizeof(double), h->m * sizeof(double), group_cols(h, j),
-                                              cudaMemcpyDefault, o.s_upd));
+                CUDA_TRY(h, cudaMemcpy2DAsync(static_cast<char*>(A) + j * nb * lda * es, lda * es,
+                                              h->at(o.io, (int64_t)lc * h->m * nb), h->m * es, h->m * es,
+                                              group_cols(h, j), cudaMemcpyDefault, o.s_upd));
             }
         }
     }
@@ -792,55 +865,52 @@ static tqr_status single_device(tqr_plan h, int* dev) {
     return TQR_OK;
 }
 
-static tqr_status apply_device(tqr_plan h, char trans, double* Bw, int64_t ldw, int64_t nslices, cudaStream_t s) {
-    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
-    const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile;
+// Bw (mp x 32*nslices, ld ldw) <- Q^T Bw (forward over the panels) or Q Bw (reverse).
+static tqr_status apply_device(tqr_plan h, char trans, void* Bw, int64_t ldw, int64_t nslices, cudaStream_t s) {
+    const int q = h->q, nb = h->nb;
     const bool fwd = (trans == 'T' || trans == 't');
     for (int s_ = 0; s_ < q; ++s_) {
         const int k = fwd ? s_ : q - 1 - s_;
         Owner* O = h->local(h->owner_of[k]);
-        const int lc = O->lidx[k];
-        UpdateArgs u;
-        u.V = O->Vimg + lc * colsz; u.T = O->T + lc * (int64_t)p * tsz; u.Vexp = O->Vexp + lc * tile;
-        u.X = Bw; u.col_stride = (int64_t)nb * ldw; u.tile_stride = nb; u.ld = ldw;
-        u.group0 = 0; u.gstride = 1; u.k = k; u.p = p; u.do_unmqr = 1;
-        CUDA_TRY(h, tqr::launch_update(nb, ib, 32, u, (int)nslices, fwd, s));
+        const PanelRefs r = own_refs(h, *O, O->lidx[k]);
+        CUDA_TRY(h, update(h, r, Bw, (int64_t)nb * ldw, nb, ldw, 0, 1, k, 32, (int)nslices, fwd, s));
         h->launches++;
     }
     return TQR_OK;
 }
 
-static tqr_status stage_b(tqr_plan h, const double* B, int64_t ldb, int64_t nrhs, int64_t* nslices, cudaStream_t s) {
+// Stage B (m x nrhs) into the zero-padded workspace (mp x nrhs rounded up to 32 columns).
+static tqr_status stage_b(tqr_plan h, const void* B, int64_t ldb, int64_t nrhs, int64_t* nslices, cudaStream_t s) {
     const int64_t pad = (nrhs + 31) / 32 * 32;
     *nslices = pad / 32;
     const int64_t mp = (int64_t)h->p * h->nb;   // zero-padded rows m..mp-1 (Q = diag(Q_m, I))
     const size_t need = (size_t)mp * pad;
+    const size_t es = h->es;
     if (need > h->bw_elems) {
         if (h->bw) cudaFree(h->bw);
         h->bw = nullptr;
         h->bw_elems = 0;
-        CUDA_TRY(h, cudaMalloc(&h->bw, need * sizeof(double)));
+        CUDA_TRY(h, cudaMalloc(&h->bw, need * es));
         h->bw_elems = need;
     }
-    CUDA_TRY(h, cudaMemsetAsync(h->bw, 0, need * sizeof(double), s));
-    CUDA_TRY(h, cudaMemcpy2DAsync(h->bw, mp * sizeof(double), B, ldb * sizeof(double), h->m * sizeof(double), nrhs,
-                                  cudaMemcpyDefault, s));
+    CUDA_TRY(h, cudaMemsetAsync(h->bw, 0, need * es, s));
+    CUDA_TRY(h, cudaMemcpy2DAsync(h->bw, mp * es, B, ldb * es, h->m * es, nrhs, cudaMemcpyDefault, s));
     return TQR_OK;
 }
 
-tqr_status tqr_apply_qt(tqr_plan h, char trans, void* Bv, int64_t ldb, int64_t nrhs) {
+tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "apply_qt before a successful factor");
     if (!(trans == 'T' || trans == 't' || trans == 'N' || trans == 'n')) return fail(h, TQR_ERR_ARG, "trans must be 'T' or 'N'");
-    if (nrhs < 0 || (nrhs > 0 && (!Bv || ldb < h->m))) return fail(h, TQR_ERR_ARG, "apply_qt: bad B/ldb/nrhs");
+    if (nrhs < 0 || (nrhs > 0 && (!B || ldb < h->m))) return fail(h, TQR_ERR_ARG, "apply_qt: bad B/ldb/nrhs");
     if (nrhs == 0) return TQR_OK;
     int dev = 0;
     tqr_status st = single_device(h, &dev);
     if (st) return st;
     CUDA_TRY(h, cudaSetDevice(dev));
     cudaStream_t s = h->owners[0].s_upd;
-    double* B = static_cast<double*>(Bv);
+    const size_t es = h->es;
     st = sync_entry(h, classify(B));
     if (st) return st;
     int64_t nsl = 0;
@@ -849,24 +919,23 @@ tqr_status tqr_apply_qt(tqr_plan h, char trans, void* Bv, int64_t ldb, int64_t n
     const int64_t mp = (int64_t)h->p * h->nb;
     st = apply_device(h, trans, h->bw, mp, nsl, s);
     if (st) return st;
-    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, mp * sizeof(double), h->m * sizeof(double), nrhs,
-                                  cudaMemcpyDefault, s));
+    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * es, h->bw, mp * es, h->m * es, nrhs, cudaMemcpyDefault, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     return TQR_OK;
 }
 
-tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
+tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "solve_ls before a successful factor");
-    if (nrhs < 0 || (nrhs > 0 && (!Bv || ldb < h->m))) return fail(h, TQR_ERR_ARG, "solve_ls: bad B/ldb/nrhs");
+    if (nrhs < 0 || (nrhs > 0 && (!B || ldb < h->m))) return fail(h, TQR_ERR_ARG, "solve_ls: bad B/ldb/nrhs");
     if (nrhs == 0) return TQR_OK;
     int dev = 0;
     tqr_status st = single_device(h, &dev);
     if (st) return st;
     CUDA_TRY(h, cudaSetDevice(dev));
     cudaStream_t s = h->owners[0].s_upd;
-    double* B = static_cast<double*>(Bv);
+    const size_t es = h->es;
     st = sync_entry(h, classify(B));
     if (st) return st;
     int64_t nsl = 0;
@@ -876,26 +945,26 @@ tqr_status tqr_solve_ls(tqr_plan h, void* Bv, int64_t ldb, int64_t nrhs) {
     st = apply_device(h, 'T', h->bw, mp, nsl, s);
     if (st) return st;
     // gather R (n x n, column-major) from every owner
-    const int64_t n = h->n, nb = h->nb, tile = nb * nb;
-    if (!h->rcm) CUDA_TRY(h, cudaMalloc(&h->rcm, sizeof(double) * (size_t)n * n));
+    const int64_t n = h->n, nb = h->nb;
+    if (!h->rcm) CUDA_TRY(h, cudaMalloc(&h->rcm, es * (size_t)n * n));
     if (!h->dflag) CUDA_TRY(h, cudaMalloc(&h->dflag, sizeof(int64_t)));
     for (auto& o : h->owners) {
         if (o.cols.empty()) continue;
-        CUDA_TRY(h, tqr::launch_from_tiles(h->rcm, n, nb * n, o.tiles, o.cols_dev, (int)o.cols.size(), h->p * tile,
-                                           (int)nb, n, n, 0, s));
+        CUDA_TRY(h, from_tiles(h, h->rcm, n, nb * n, o.tiles, o.cols_dev, (int)o.cols.size(), n, n, 0, s));
         h->launches++;
     }
     const int64_t big = INT64_MAX;
     CUDA_TRY(h, cudaMemcpyAsync(h->dflag, &big, sizeof(int64_t), cudaMemcpyHostToDevice, s));
-    CUDA_TRY(h, tqr::launch_zero_diag_check(h->rcm, n, n, h->dflag, s));
+    if (h->f32()) CUDA_TRY(h, tqr::launch_zero_diag_check<float>((const float*)h->rcm, n, n, h->dflag, s));
+    else CUDA_TRY(h, tqr::launch_zero_diag_check<double>((const double*)h->rcm, n, n, h->dflag, s));
     int64_t first_zero = 0;
     CUDA_TRY(h, cudaMemcpyAsync(&first_zero, h->dflag, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     if (first_zero != big) return fail(h, TQR_ERR_SINGULAR, "R(%lld,%lld) == 0", (long long)first_zero, (long long)first_zero);
-    CUDA_TRY(h, tqr::launch_trsv_upper(h->rcm, n, h->bw, mp, n, nrhs, s));
+    if (h->f32()) CUDA_TRY(h, tqr::launch_trsv_upper<float>((const float*)h->rcm, n, (float*)h->bw, mp, n, nrhs, s));
+    else CUDA_TRY(h, tqr::launch_trsv_upper<double>((const double*)h->rcm, n, (double*)h->bw, mp, n, nrhs, s));
     h->launches++;
-    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * sizeof(double), h->bw, mp * sizeof(double), n * sizeof(double), nrhs,
-                                  cudaMemcpyDefault, s));
+    CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * es, h->bw, mp * es, n * es, nrhs, cudaMemcpyDefault, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     return TQR_OK;
 }

@@ -19,12 +19,13 @@ struct PanelArgs {
 };
 
 // Trailing update of step k over `ngroups` column groups (UNMQR + TSMQR chain), or the
-// application of panel k's Q^T / Q to a right-hand side block (tqr_apply_qt).
-struct UpdateArgs {
-    const double* V;     // stage images of panel k's reflector tiles: tile i at V + i*nb*nb (i > k used)
-    const double* Vexp;  // stage image of the explicit V of the diagonal tile
-    const double* T;     // T factors: tile i at T + i*ib*nb
-    double* X;           // target: element (tile i, r, c) of group gidx at
+// application of panel k's Q^T / Q to a right-hand side block (tqr_apply_qt).  T = element type.
+template <class E>
+struct UpdateArgsT {
+    const E* V;          // stage images of panel k's reflector tiles (tile i at V + i*image tile, i > k used)
+    const E* Vexp;       // stage image of the explicit V of the diagonal tile
+    const E* T;          // T factors: tile i at T + i*ib*nb
+    E* X;                // target: element (tile i, r, c) of group gidx at
                          //   X + gidx*col_stride + i*tile_stride + c*ld + r
     int64_t col_stride;
     int64_t tile_stride;
@@ -34,6 +35,7 @@ struct UpdateArgs {
     int k, p;
     int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
 };
+using UpdateArgs = UpdateArgsT<double>;
 
 // split = apply CTAs per ib column block (1, 2, 4): grid = (nb/ib) * (split + 1)
 cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s);
@@ -52,9 +54,21 @@ template <class T>
 cudaError_t launch_from_tiles(T* dst, int64_t lda, int64_t dst_group_stride, const T* src, const int32_t* cols_dev,
                               int ncols, int64_t src_col_stride, int nb, int64_t m_rows, int64_t n_valid,
                               int local_dst, cudaStream_t s);
-cudaError_t launch_trsv_upper(const double* R, int64_t ldr, double* C, int64_t ldc, int64_t n, int64_t nrhs,
+template <class T>
+cudaError_t launch_trsv_upper(const T* R, int64_t ldr, T* C, int64_t ldc, int64_t n, int64_t nrhs, cudaStream_t s);
+template <class T>
+cudaError_t launch_zero_diag_check(const T* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s);
+
+// ---- FP32 path (kernels/qr_kernels_f32.cu)
+// FFMA trailing update; V / Vexp are FP32 stage images (f32_img_tile elements per tile)
+cudaError_t launch_update_f32(int nb, int ib, int w, const UpdateArgsT<float>& a, int nslices, bool trans,
                               cudaStream_t s);
-cudaError_t launch_zero_diag_check(const double* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s);
+// FP32 -> FP64 copy of n elements (n % 4 == 0, 16-byte aligned)
+cudaError_t launch_widen(const float* src, double* dst, int64_t n, cudaStream_t s);
+// FP64 panel result of step k (scratch column sc, T64) -> FP32 tiles, T and stage images
+cudaError_t launch_narrow_panel(int nb, int ib, const double* sc, const double* T64, float* tiles, float* T32,
+                                float* Vimg, float* Vexp, int k, int p, cudaStream_t s);
+int64_t f32_img_tile(int nb, int ib);
 size_t panel_smem_bytes(int nb, int ib);
 size_t update_smem_bytes(int nb, int ib, int w);
 
