@@ -53,12 +53,8 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel32(UpdateArgsT<float
             const float* nxt = nullptr;
             if (si + 1 < NBLK) nxt = vblock(ti, blk(si + 1));
             else if (q + 1 < ntiles) nxt = vblock(tile_of(q + 1), blk(0));
-            if (ti < 0)
-                apply_block32<NB, W, IB, TRANS, true>(X, sm, Tt + (int64_t)s * IB * IB, nullptr, a.ld, s * IB, nxt,
-                                                      vph, buf);
-            else
-                apply_block32<NB, W, IB, TRANS, false>(X, sm, Tt + (int64_t)s * IB * IB, Xk + s * IB, a.ld, 0, nxt,
-                                                       vph, buf);
+            apply_block32<NB, W, IB, TRANS>(X, sm, Tt + (int64_t)s * IB * IB, ti < 0 ? nullptr : Xk + s * IB, a.ld,
+                                            ti < 0 ? s * IB : 0, nxt, vph, buf);
         }
         X.store(Xi, a.ld);
         __syncthreads();   // row tile k (the TS "top") is re-read by other threads
@@ -115,6 +111,9 @@ __global__ void __launch_bounds__(256) narrow_panel_kernel(const double* __restr
 
 template <int NB, int W, int IB>
 static cudaError_t launch_update32_t(const UpdateArgsT<float>& a, int nslices, bool trans, cudaStream_t s) {
+  if constexpr (!G32<NB, W, IB>::ok) {
+    return cudaErrorInvalidValue;     // slice too narrow for the tile (nb = 64, w = 8)
+  } else {
     const size_t smem = sizeof(Smem32<NB, W, IB>);
     if (nslices <= 0) return cudaSuccess;
     if (trans) {
@@ -129,13 +128,19 @@ static cudaError_t launch_update32_t(const UpdateArgsT<float>& a, int nslices, b
         kern<<<nslices, kThreads, smem, s>>>(a);
     }
     return cudaGetLastError();
+  }
 }
 
 constexpr size_t kMaxSmem = 232448;
-#define TQR_FITS32(NB_, IB_)                                                         \
-    static_assert(sizeof(Smem32<NB_, 8, IB_>) <= kMaxSmem, "f32 update smem W=8");   \
-    static_assert(sizeof(Smem32<NB_, 16, IB_>) <= kMaxSmem, "f32 update smem W=16"); \
-    static_assert(sizeof(Smem32<NB_, 32, IB_>) <= kMaxSmem, "f32 update smem W=32");
+template <int NB, int W, int IB>
+constexpr bool fits() {
+    if constexpr (G32<NB, W, IB>::ok) return sizeof(Smem32<NB, W, IB>) <= kMaxSmem;
+    else return true;
+}
+#define TQR_FITS32(NB_, IB_)                                                \
+    static_assert(fits<NB_, 8, IB_>(), "f32 update smem W=8");              \
+    static_assert(fits<NB_, 16, IB_>(), "f32 update smem W=16");            \
+    static_assert(fits<NB_, 32, IB_>(), "f32 update smem W=32");
 TQR_FITS32(64, 16) TQR_FITS32(64, 32) TQR_FITS32(128, 16) TQR_FITS32(128, 32)
 TQR_FITS32(256, 16) TQR_FITS32(256, 32) TQR_FITS32(512, 16) TQR_FITS32(512, 32)
 #undef TQR_FITS32

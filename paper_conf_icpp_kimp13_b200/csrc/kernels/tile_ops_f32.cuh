@@ -9,9 +9,11 @@
 //     X1 -= W' ;  X -= V_s W'     (GEMM2, K = ib)
 // sm_100a has no FP32-accurate tensor-core kind (TF32 keeps 10 mantissa bits, too few for the
 // 1e-5 residual bar), so both GEMMs are FFMA: thread (rg, cg) of warp w owns the R = RW/RG rows
-// w*RW + rg + RG*i (interleaved) of the column pair (2cg, 2cg+1).  Every 16-byte shared-memory
-// read of V (4 consecutive k of one row, broadcast to the CG lanes sharing the row) feeds 8 FFMAs
-// in both GEMMs.  V is staged per warp (each warp only reads its own RW rows) by one
+// w*RW + rg + RG*i (interleaved) of the column quad 4cg..4cg+3.  Every 16-byte shared-memory
+// read of V (4 consecutive k of one row, broadcast to the CG lanes sharing the row) feeds 16 FFMAs
+// in both GEMMs, which keeps the shared-memory pipe (2 wavefronts per such read: one per
+// half-warp) below the FFMA pipe (measured: 2 columns per thread made the kernel smem-bound).
+// GEMM1 runs in k-chunks of 16 so the partial sums fit in registers next to X.  V is staged per warp (each warp only reads its own RW rows) by one
 // cp.async.bulk from the "stage image" the panel step writes: block s of a tile is NB rows of
 // IBP = IB + 4 floats (k contiguous, 4 floats of padding), so the RG adjacent rows read together
 // fall in distinct 16-byte bank groups without a swizzle.  Two buffers per warp: block s+1 is in
@@ -28,16 +30,18 @@ constexpr int kWarps = 8;
 template <int NB, int W, int IB>
 struct G32 {
     static constexpr int RW = NB / kWarps;      // rows per warp
-    static constexpr int CG = W / 2;            // column pairs (lanes & (CG-1))
+    static constexpr int CG = W / 4;            // column quads (lanes % CG)
     static constexpr int RG = 32 / CG;          // row groups per warp
     static constexpr int R = RW / RG;           // rows per thread
     static constexpr int KC = IB / 4;           // 16-byte chunks per V row
+    static constexpr int KCH = 16;              // GEMM1 k-chunk
+    static constexpr int NCH = IB / KCH;        // GEMM1 chunks
+    static constexpr int KPL = KCH / RG;        // k values per lane and chunk after the reduce-scatter
     static constexpr int IBP = IB + 4;          // padded V row (floats)
     static constexpr int VBLK = RW * IBP;       // one warp's staged rows of one block (floats)
-    static constexpr int KR = IB / RG;          // k values per lane after the reduce-scatter
     static constexpr int LDT = IB + 4;          // Tsm / topsm row pitch (16-byte aligned, bank-skewed)
     static constexpr int W4 = W / 4;            // float4 column groups in the reduction
-    static_assert(W % 8 == 0 && 32 % CG == 0 && R >= 1 && IB % RG == 0 && IB % 4 == 0, "geometry");
+    static constexpr bool ok = (W % 8 == 0) && (32 % CG == 0) && (RW >= RG) && (KCH % RG == 0) && (IB % KCH == 0);
     static_assert(IB * W4 <= kThreads, "reduction mapping");
 };
 
@@ -53,6 +57,7 @@ __host__ __device__ __forceinline__ int64_t img_off(int r, int c) {
 
 template <int NB, int W, int IB>
 struct Smem32 {
+    static_assert(G32<NB, W, IB>::ok, "f32 geometry");
     using G = G32<NB, W, IB>;
     uint64_t mbar[kWarps][2];                   // bulk-copy completion of vbuf[w][b]
     float vbuf[kWarps][2][G::VBLK];
@@ -66,23 +71,21 @@ struct Smem32 {
 template <int NB, int W, int IB>
 struct Slice32 {
     using G = G32<NB, W, IB>;
-    float x[G::R][2];
+    float x[G::R][4];
     // element (r, c) of the slice at P[c*ld + r]
     __device__ __forceinline__ void load(const float* P, int64_t ld) {
         const int lane = lane_id(), cg = lane % G::CG, rg = lane / G::CG, rb = warp_id() * G::RW + rg;
 #pragma unroll
-        for (int i = 0; i < G::R; ++i) {
-            x[i][0] = P[(int64_t)(2 * cg) * ld + rb + G::RG * i];
-            x[i][1] = P[(int64_t)(2 * cg + 1) * ld + rb + G::RG * i];
-        }
+        for (int i = 0; i < G::R; ++i)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) x[i][c] = P[(int64_t)(4 * cg + c) * ld + rb + G::RG * i];
     }
     __device__ __forceinline__ void store(float* P, int64_t ld) const {
         const int lane = lane_id(), cg = lane % G::CG, rg = lane / G::CG, rb = warp_id() * G::RW + rg;
 #pragma unroll
-        for (int i = 0; i < G::R; ++i) {
-            P[(int64_t)(2 * cg) * ld + rb + G::RG * i] = x[i][0];
-            P[(int64_t)(2 * cg + 1) * ld + rb + G::RG * i] = x[i][1];
-        }
+        for (int i = 0; i < G::R; ++i)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) P[(int64_t)(4 * cg + c) * ld + rb + G::RG * i] = x[i][c];
     }
 };
 
@@ -113,15 +116,16 @@ __device__ __forceinline__ void stage32(Smem32<NB, W, IB>& sm, const float* blk,
 //   next : image of the following block (staged here into vbuf[w][buf^1]) or null.
 //   Ts   : T block (IB x IB column-major, zeros below the diagonal).
 //   top  : X1 (IB x W, element (r, c) at top[c*ldtop + r]) or null (UNMQR).
-//   KM   : rows < kmin of V are zero; warps whose rows are all < kmin skip both GEMMs.
-template <int NB, int W, int IB, bool TRANS, bool KM>
+//   kmin : rows < kmin of V are zero (UNMQR blocks); warps whose rows are all < kmin skip both
+//          GEMMs.  A runtime value (not a template flag) so the kernel holds one copy of this body.
+template <int NB, int W, int IB, bool TRANS>
 __device__ __forceinline__ void apply_block32(Slice32<NB, W, IB>& X, Smem32<NB, W, IB>& sm,
                                               const float* __restrict__ Ts, float* top, int64_t ldtop,
                                               int kmin, const float* next, unsigned& vph, int& buf) {
     using G = G32<NB, W, IB>;
     const int lane = lane_id(), w = warp_id(), tid = threadIdx.x;
     const int cg = lane % G::CG, rg = lane / G::CG;
-    const bool active = !KM || (w + 1) * G::RW > kmin;
+    const bool active = (w + 1) * G::RW > kmin;
 
     // ---- (0) T block and X1 rows (LDGSTS, waited before barrier 1); next block's V (bulk)
     for (int id = tid; id < IB * IB / 4; id += kThreads) {
@@ -140,50 +144,55 @@ __device__ __forceinline__ void apply_block32(Slice32<NB, W, IB>& X, Smem32<NB, 
     if (next) stage32(sm, next, buf ^ 1);
     const float* vb = &sm.vbuf[w][buf][0];
 
-    // ---- (1) GEMM1: P(k, c) = sum over my rows of V(r, k) X(r, c)
-    float P[IB][2];
+    // ---- (1) GEMM1 per k-chunk: P(k, c) = sum over my rows of V(r, k) X(r, c), then a
+    //      reduce-scatter over the RG lanes sharing a column quad (xor 16, 8, .., CG): each level
+    //      halves the k range a lane keeps; one float4 store per kept k
+#pragma unroll 1
+    for (int ch = 0; ch < G::NCH; ++ch) {     // runtime loop: keeps the body in the instruction cache
+        float P[G::KCH][4];
 #pragma unroll
-    for (int k = 0; k < IB; ++k) P[k][0] = P[k][1] = 0.f;
-    if (active) {
+        for (int k = 0; k < G::KCH; ++k)
 #pragma unroll
-        for (int i = 0; i < G::R; ++i) {
-            const float4* vr = reinterpret_cast<const float4*>(vb + (rg + G::RG * i) * G::IBP);
-            const float x0 = X.x[i][0], x1 = X.x[i][1];
+            for (int c = 0; c < 4; ++c) P[k][c] = 0.f;
+        if (active) {
 #pragma unroll
-            for (int kc = 0; kc < G::KC; ++kc) {
-                const float4 v = vr[kc];
-                P[4 * kc + 0][0] = fmaf(v.x, x0, P[4 * kc + 0][0]);
-                P[4 * kc + 0][1] = fmaf(v.x, x1, P[4 * kc + 0][1]);
-                P[4 * kc + 1][0] = fmaf(v.y, x0, P[4 * kc + 1][0]);
-                P[4 * kc + 1][1] = fmaf(v.y, x1, P[4 * kc + 1][1]);
-                P[4 * kc + 2][0] = fmaf(v.z, x0, P[4 * kc + 2][0]);
-                P[4 * kc + 2][1] = fmaf(v.z, x1, P[4 * kc + 2][1]);
-                P[4 * kc + 3][0] = fmaf(v.w, x0, P[4 * kc + 3][0]);
-                P[4 * kc + 3][1] = fmaf(v.w, x1, P[4 * kc + 3][1]);
+            for (int i = 0; i < G::R; ++i) {
+                const float4* vr = reinterpret_cast<const float4*>(vb + (rg + G::RG * i) * G::IBP + ch * G::KCH);
+                float4 v[G::KCH / 4];
+#pragma unroll
+                for (int q = 0; q < G::KCH / 4; ++q) v[q] = vr[q];
+#pragma unroll
+                for (int q = 0; q < G::KCH / 4; ++q)
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) {
+                        const float xc = X.x[i][c];
+                        P[4 * q + 0][c] = fmaf(v[q].x, xc, P[4 * q + 0][c]);
+                        P[4 * q + 1][c] = fmaf(v[q].y, xc, P[4 * q + 1][c]);
+                        P[4 * q + 2][c] = fmaf(v[q].z, xc, P[4 * q + 2][c]);
+                        P[4 * q + 3][c] = fmaf(v[q].w, xc, P[4 * q + 3][c]);
+                    }
             }
         }
+        int k0 = ch * G::KCH;
+#pragma unroll
+        for (int j = 0; (1 << j) < G::RG; ++j) {
+            const int m = 16 >> j;
+            const int H = (G::KCH >> j) / 2;
+            const bool up = (lane & m) != 0;
+#pragma unroll
+            for (int e = 0; e < H; ++e)
+#pragma unroll
+                for (int c = 0; c < 4; ++c) {
+                    const float send = up ? P[e][c] : P[e + H][c];
+                    const float keep = up ? P[e + H][c] : P[e][c];
+                    P[e][c] = keep + __shfl_xor_sync(0xffffffffu, send, m);
+                }
+            if (up) k0 += H;
+        }
+#pragma unroll
+        for (int e = 0; e < G::KPL; ++e)
+            *reinterpret_cast<float4*>(&sm.red[w][k0 + e][4 * cg]) = make_float4(P[e][0], P[e][1], P[e][2], P[e][3]);
     }
-    // ---- (2) reduce-scatter over the RG lanes sharing a column pair (xor 16, 8, .., CG): each
-    //      level halves the k range a lane keeps; then one float2 store per kept k
-    int k0 = 0;
-#pragma unroll
-    for (int j = 0; (1 << j) < G::RG; ++j) {
-        const int m = 16 >> j;
-        const int H = (IB >> j) / 2;
-        const bool up = (lane & m) != 0;
-#pragma unroll
-        for (int e = 0; e < H; ++e)
-#pragma unroll
-            for (int c = 0; c < 2; ++c) {
-                const float send = up ? P[e][c] : P[e + H][c];
-                const float keep = up ? P[e + H][c] : P[e][c];
-                P[e][c] = keep + __shfl_xor_sync(0xffffffffu, send, m);
-            }
-        if (up) k0 += H;
-    }
-#pragma unroll
-    for (int e = 0; e < G::KR; ++e)
-        *reinterpret_cast<float2*>(&sm.red[w][k0 + e][2 * cg]) = make_float2(P[e][0], P[e][1]);
     cp_async_wait<0>();
     __syncthreads();
 
@@ -222,21 +231,20 @@ __device__ __forceinline__ void apply_block32(Slice32<NB, W, IB>& X, Smem32<NB, 
 
     // ---- (5) GEMM2: X(r, c) += sum_k V(r, k) Wn(k, c)
     if (active) {
+#pragma unroll 1
+        for (int kc = 0; kc < G::KC; ++kc) {   // runtime loop (instruction-cache footprint)
+            float4 wv[4];
 #pragma unroll
-        for (int kc = 0; kc < G::KC; ++kc) {
-            float2 wv[4];
-#pragma unroll
-            for (int e = 0; e < 4; ++e) wv[e] = *reinterpret_cast<const float2*>(&sm.Wn[4 * kc + e][2 * cg]);
+            for (int e = 0; e < 4; ++e) wv[e] = *reinterpret_cast<const float4*>(&sm.Wn[4 * kc + e][4 * cg]);
 #pragma unroll
             for (int i = 0; i < G::R; ++i) {
                 const float4 v = reinterpret_cast<const float4*>(vb + (rg + G::RG * i) * G::IBP)[kc];
-                float a0 = X.x[i][0], a1 = X.x[i][1];
-                a0 = fmaf(v.x, wv[0].x, a0); a1 = fmaf(v.x, wv[0].y, a1);
-                a0 = fmaf(v.y, wv[1].x, a0); a1 = fmaf(v.y, wv[1].y, a1);
-                a0 = fmaf(v.z, wv[2].x, a0); a1 = fmaf(v.z, wv[2].y, a1);
-                a0 = fmaf(v.w, wv[3].x, a0); a1 = fmaf(v.w, wv[3].y, a1);
-                X.x[i][0] = a0;
-                X.x[i][1] = a1;
+                float a0 = X.x[i][0], a1 = X.x[i][1], a2 = X.x[i][2], a3 = X.x[i][3];
+                a0 = fmaf(v.x, wv[0].x, a0); a1 = fmaf(v.x, wv[0].y, a1); a2 = fmaf(v.x, wv[0].z, a2); a3 = fmaf(v.x, wv[0].w, a3);
+                a0 = fmaf(v.y, wv[1].x, a0); a1 = fmaf(v.y, wv[1].y, a1); a2 = fmaf(v.y, wv[1].z, a2); a3 = fmaf(v.y, wv[1].w, a3);
+                a0 = fmaf(v.z, wv[2].x, a0); a1 = fmaf(v.z, wv[2].y, a1); a2 = fmaf(v.z, wv[2].z, a2); a3 = fmaf(v.z, wv[2].w, a3);
+                a0 = fmaf(v.w, wv[3].x, a0); a1 = fmaf(v.w, wv[3].y, a1); a2 = fmaf(v.w, wv[3].z, a2); a3 = fmaf(v.w, wv[3].w, a3);
+                X.x[i][0] = a0; X.x[i][1] = a1; X.x[i][2] = a2; X.x[i][3] = a3;
             }
         }
     }
