@@ -306,6 +306,26 @@ def main():
         # one step overlap, so a per-launch average duration would not be a kernel duration)
         achieved = (uflops / (ums * 1e-3) / 1e12) if ucount else None
         prof = load_profile_summary(args.config + ("_f32" if f32 else ""))
+        if ucount and ums >= pms:
+            # dominant kernel: the bulk trailing update
+            roofline = {"bound": "alu" if f32 else "tensor",
+                        "kernel": "update_kernel32<%d,32,%d> (UNMQR+TSMQR chain, FFMA)" % (nb, ib) if f32 else
+                        "update_kernel<%d,32,%d> (UNMQR+TSMQR chain, DMMA.8x8x4)" % (nb, ib),
+                        "achieved": round(achieved, 3), "peak": peak, "unit": "TFLOP/s",
+                        "frac": round(achieved / peak, 4),
+                        "traffic": prof.get("dram_bytes_per_launch"), "traffic_note": prof.get("note"),
+                        "peak_source": peak_src, "launches_per_step": ucount // K,
+                        "busy_ms_per_step": round(ums / K, 3), "share_of_step": round(ums / K / ms, 3)}
+        else:
+            # dominant kernel: the panel step (C4: one column -> the whole factorisation is panel
+            # work: TS-domain kernel + TT merge chain in tree mode, DMMA.8x8x4)
+            pach = pflops / max(pms, 1e-9) / 1e9
+            roofline = {"bound": "alu" if f32 else "tensor",
+                        "kernel": "panel step (domain_kernel<%d,%d> + merge panel_kernel, DMMA.8x8x4)" % (nb, ib),
+                        "achieved": round(pach, 3), "peak": peak, "unit": "TFLOP/s", "frac": round(pach / peak, 4),
+                        "traffic": prof.get("dram_bytes_per_launch"), "traffic_note": prof.get("note"),
+                        "peak_source": peak_src, "launches_per_step": pcount // K,
+                        "busy_ms_per_step": round(pms / K, 3), "share_of_step": round(pms / K / ms, 3)}
         line = {
             "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak",
             "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
@@ -317,16 +337,7 @@ def main():
                        "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
                        "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (es * m * n / 2 ** 30)
                        if es * m * n > L2_BYTES else "input fits L2 (no flush)"},
-            "roofline": {"bound": "alu" if f32 else "tensor",
-                         "kernel": "update_kernel32<512,32,32> (UNMQR+TSMQR chain, FFMA)" if f32 else
-                         "update_kernel<512,32,32> (UNMQR+TSMQR chain, DMMA.8x8x4)",
-                         "achieved": round(achieved, 3) if achieved else None, "peak": peak, "unit": "TFLOP/s",
-                         "frac": round(achieved / peak, 4) if achieved else None,
-                         "traffic": prof.get("dram_bytes_per_launch"),
-                         "traffic_note": prof.get("note"),
-                         "peak_source": peak_src, "launches_per_step": ucount // K,
-                         "busy_ms_per_step": round(ums / K, 3),
-                         "share_of_step": round(ums / K / ms, 3) if ucount else None},
+            "roofline": roofline,
             "panel": {"launches": pcount, "avg_ms": round(pms / max(pcount, 1), 3),
                       "tflops": round(pflops / max(pms, 1e-9) / 1e9, 3) if pcount else None},
             "clocks": clk.summary(),

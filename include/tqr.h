@@ -66,6 +66,12 @@ typedef struct {
     /* 1: record CUDA events around every update-kernel launch so tqr_kernel_stats() can
      * report the dominant kernel's device time (bench.py roofline). */
     int32_t profile;
+    /* Elimination tree (the paper's TT elimination): every panel
+     * column is split into TS domains of L tiles, each factored (GEQRT of its head + TSQRT chain)
+     * by one CTA concurrently, and the domain heads' R factors are merged by a TT chain; updates
+     * and tqr_apply_qt replay the same tree.  0 = auto (tree for a single column tile, q == 1,
+     * with L = ceil(p / SM count)), -1 = always flat TS, L > 0 = domains of L tiles (FP64 only). */
+    int32_t tree_domain;
 } tqr_options;
 
 /*

@@ -62,7 +62,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     const bool leader = (u == S);              // the factor CTA of block b
     const int64_t tile = (int64_t)NB * NB;
     double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
-    double* Akk = col + (int64_t)a.k * tile;
+    double* Akk = a.top ? a.top : col + (int64_t)a.k * tile;
     unsigned* F = a.flags;                                   // p * NBLK
     unsigned* Gf = a.flags + (int64_t)a.p * NBLK;            // p * NBLK * S
     const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
@@ -70,7 +70,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     stage_init(sa);
     TQR_PP0();
 
-    for (int i = a.k; i < a.p; ++i) {
+    for (int i = a.k + a.skip_ge; i < a.p; ++i) {
         double* Ai = col + (int64_t)i * tile;
         double* Ti = a.T + (int64_t)i * IB * NB;
         const bool ge = (i == a.k);
@@ -163,6 +163,107 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         if (threadIdx.x == 0) flag_release(F + (int64_t)i * NBLK + b, a.epoch);
         TQR_TRACE("cta %d (b%d u%d) tile %d published F\n", blockIdx.x, b, u, i);
         TQR_PP(3);
+    }
+}
+
+// ============================================================================ domain kernel
+// TS-domain factorisation (tree mode): one CTA per domain, which runs the whole GEQRT(head) +
+// TSQRT(i, head) chain of its tiles alone -- per tile and ib column block b: the block's NB x IB
+// columns in registers, the b earlier reflector blocks of the same tile applied (apply_block,
+// DMMA), then factor_block -- with no inter-CTA flags.  Many domains run at once (one per SM),
+// which is what the flat chain of a tall panel lacks (C4: parallelism 1).
+template <int NB, int IB>
+__global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    auto& sf = *reinterpret_cast<Smem<NB, IB, IB, true>*>(smem_raw);
+    using G = Geom<NB, IB, IB>;
+    constexpr int NBLK = NB / IB;
+    const int64_t tile = (int64_t)NB * NB;
+    const int head = a.k + blockIdx.x * a.L;
+    const int end = min(head + a.L, a.p);
+    double* Ah = a.col + (int64_t)head * tile;
+    double* himg = (head == a.k) ? a.Vexp : a.Vimg + (int64_t)head * tile;
+    const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
+    unsigned vph = 0;
+    stage_init(sf);
+    for (int i = head; i < end; ++i) {
+        double* Ai = a.col + (int64_t)i * tile;
+        double* Ti = a.T + (int64_t)i * IB * NB;
+        const bool ge = (i == head);
+        double* img = ge ? himg : a.Vimg + (int64_t)i * tile;
+        for (int b = 0; b < NBLK; ++b) {
+            Slice<NB, IB, IB> X;
+            X.load_cg(Ai + (int64_t)b * IB * NB, NB);
+            for (int bp = 0; bp < b; ++bp) {
+                const double* Vb = img + (int64_t)bp * IB * NB;
+                const double* nxt = (bp + 1 < b) ? img + (int64_t)(bp + 1) * IB * NB : nullptr;
+                if (bp == 0) {
+                    if (lane_id() == 0) fence_proxy_async_global();   // this CTA's image stores -> bulk copy
+                    stage_first(sf, Vb);
+                }
+                if (ge)
+                    apply_block<NB, IB, IB, true, true, true, true>(X, sf, Vb, Ti + (int64_t)bp * IB * IB, nullptr, 0,
+                                                                   bp * IB, nxt, vph);
+                else
+                    apply_block<NB, IB, IB, true, true, true, false>(X, sf, Vb, Ti + (int64_t)bp * IB * IB,
+                                                                    Ah + (int64_t)b * IB * NB + bp * IB, NB, 0, nxt,
+                                                                    vph);
+            }
+            __syncthreads();   // top rows written by the applies -> Rsm reads below
+            if (ge) {
+                factor_block<NB, IB, true>(X, sf, b * IB);
+            } else {
+                for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+                    const int c = idx / IB, j = idx % IB;
+                    sf.Rsm[c * IB + j] = (j >= c) ? ld_cg(Ah + (int64_t)(b * IB + j) * NB + b * IB + c) : 0.0;
+                }
+                __syncthreads();
+                factor_block<NB, IB, false>(X, sf, b * IB);
+            }
+            X.store(Ai + (int64_t)b * IB * NB, NB);
+#pragma unroll
+            for (int mf = 0; mf < IB / 8; ++mf) {
+                const int cb = mf * 8 + g;
+                const int dc = b * IB + cb;
+#pragma unroll
+                for (int nf = 0; nf < G::NF; ++nf) {
+                    const int rl = nf * 8 + 2 * t;
+                    const int r = wq * G::RW + rl;
+                    double v0 = X.acc[mf][nf][0], v1 = X.acc[mf][nf][1];
+                    if (ge) {
+                        v0 = (r > dc) ? v0 : (r == dc ? 1.0 : 0.0);
+                        v1 = (r + 1 > dc) ? v1 : (r + 1 == dc ? 1.0 : 0.0);
+                    }
+                    st2(img + vimg_off<NB, IB, IB>(b, wq, cb / G::HC, rl, cb % G::HC), v0, v1);
+                }
+            }
+            if (!ge) {
+                for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+                    const int j = idx / IB, c = idx % IB;
+                    if (c <= j) Ah[(int64_t)(b * IB + j) * NB + b * IB + c] = sf.Rsm[c * IB + j];
+                }
+            }
+            build_T<NB, IB>(sf);
+            for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
+                const int c = idx / IB, r = idx % IB;
+                Ti[(int64_t)b * IB * IB + c * IB + r] = sf.Tsm[r * IB + c];
+            }
+            __threadfence_block();
+            __syncthreads();
+        }
+    }
+}
+
+// Mt[e] = triu(tile k + e*L of the column), zeros below the diagonal (e = 1..ndom-1): the dense
+// "bottom" of merge e, factored against the head tile k by the panel kernel (skip_ge).
+__global__ void merge_prep_kernel(const double* __restrict__ col, double* __restrict__ Mt, int nb, int k, int L) {
+    const int e = blockIdx.y + 1;
+    const int64_t tile = (int64_t)nb * nb;
+    const double* s = col + (int64_t)(k + e * L) * tile;
+    double* d = Mt + (int64_t)e * tile;
+    for (int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < tile; x += (int64_t)gridDim.x * blockDim.x) {
+        const int c = (int)(x / nb), r = (int)(x % nb);
+        d[x] = (r <= c) ? s[x] : 0.0;
     }
 }
 
@@ -361,6 +462,32 @@ cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStre
     TQR_PAN(256, 16) TQR_PAN(256, 32) TQR_PAN(512, 16) TQR_PAN(512, 32)
 #undef TQR_PAN
     return cudaErrorInvalidValue;
+}
+
+template <int NB, int IB>
+static cudaError_t launch_domains_t(const DomainArgs& a, int ndom, cudaStream_t s) {
+    const size_t smem = sizeof(Smem<NB, IB, IB, true>);
+    auto kern = domain_kernel<NB, IB>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<ndom, kThreads, smem, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_domains(int nb, int ib, const DomainArgs& a, int ndom, cudaStream_t s) {
+    if (ndom <= 0) return cudaSuccess;
+#define TQR_DOM(NB_, IB_) if (nb == NB_ && ib == IB_) return launch_domains_t<NB_, IB_>(a, ndom, s);
+    TQR_DOM(64, 16) TQR_DOM(64, 32) TQR_DOM(128, 16) TQR_DOM(128, 32)
+    TQR_DOM(256, 16) TQR_DOM(256, 32) TQR_DOM(512, 16) TQR_DOM(512, 32)
+#undef TQR_DOM
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_merge_prep(int nb, const double* col, double* Mt, int k, int L, int ndom, cudaStream_t s) {
+    if (ndom <= 1) return cudaSuccess;
+    dim3 grid(std::max(1, std::min(64, nb * nb / 2048)), ndom - 1);
+    merge_prep_kernel<<<grid, 256, 0, s>>>(col, Mt, nb, k, L);
+    return cudaGetLastError();
 }
 
 // w: slice width (8, 16, 32).  Narrow slices raise CTA count for the lookahead column.

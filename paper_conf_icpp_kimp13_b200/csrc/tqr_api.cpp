@@ -54,6 +54,12 @@ struct Owner {
     void* rb_V[2] = {nullptr, nullptr};
     unsigned* flags = nullptr;      // p * (nb/ib)
     void* io = nullptr;             // m x (nb*ncols) column-major mirror for host / remote I/O
+    // tree mode (TS domains + flat TT merge chain, NEXT-1): per owned column, Dmax merge slots
+    void* Mimg = nullptr;           // ncols * Dmax * vt   stage images of the merge reflectors (slot e)
+    void* MT = nullptr;             // ncols * Dmax * ib*nb  merge T factors
+    double* Mt = nullptr;           // Dmax * nb*nb        merge bottoms triu(R_e) -> V2 (factor scratch)
+    void* rb_M[2] = {nullptr, nullptr};
+    void* rb_MT[2] = {nullptr, nullptr};
     // FP32 plans: FP64 scratch of one panel column (the panel is factored in FP64, then narrowed)
     double* sc_col = nullptr;       // p * nb*nb
     double* sc_T = nullptr;         // p * ib*nb
@@ -90,6 +96,9 @@ struct tqr_plan_s {
     bool lookahead = true, profile = false;
     int nstreams = 4;               // bulk-update streams per owner (TQR_UPDATE_STREAMS)
     int panel_split = 1;            // sub-slice CTAs per ib column block in the panel kernel
+    int tree_L = 0;                 // TS-domain length (tiles); 0 = flat TS chain
+    int dmax = 1;                   // max domains of any step = ceil(p / tree_L)
+    int ndom(int k) const { return tree_L > 0 ? (p - k + tree_L - 1) / tree_L : 1; }
     std::vector<Owner> owners;      // in-process: ndev entries; multi-process: 1 (this rank)
     const tqr::NcclApi* nccl = nullptr;
     ncclComm_t comm = nullptr;
@@ -170,7 +179,8 @@ void free_owner(Owner& o) {
     cudaSetDevice(o.dev);
     auto F = [](void* p) { if (p) cudaFree(p); };
     F(o.cols_dev); F(o.tiles); F(o.Vimg); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
-    F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp);
+    F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp); F(o.Mimg); F(o.MT); F(o.Mt);
+    for (int s = 0; s < 2; ++s) { F(o.rb_M[s]); F(o.rb_MT[s]); }
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
     for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref})
         for (auto e : *v) if (e) cudaEventDestroy(e);
@@ -402,6 +412,17 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
+    // Tree mode (NEXT-1): TS domains of L tiles factored one per CTA, merged by a flat TT chain.
+    // Auto: a single panel column (q == 1, e.g. C4) whose flat chain has parallelism 1.
+    if (o.tree_domain > 0) h->tree_L = o.tree_domain;
+    else if (o.tree_domain == 0 && h->q == 1 && h->p >= 8) {
+        int sms = 148;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+        h->tree_L = std::max(2, (h->p + sms - 1) / sms);
+    }
+    if (h->tree_L >= h->p) h->tree_L = 0;
+    if (h->tree_L > 0 && dtype != TQR_F64) { h->tree_L = 0; if (o.tree_domain > 0) { delete h; return fail(nullptr, TQR_ERR_UNSUPPORTED, "tree mode: FP64 only in this build"); } }
+    h->dmax = h->ndom(0);
     // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
     // panel is on the critical path (few trailing columns per panel step or several owners).
     h->panel_split = (h->q <= 4) ? 4 : 2;   // measured: 4 for tall / few columns, 2 otherwise
@@ -464,6 +485,10 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         if (!alloc(&ow.tiles, nc * p * tile) || !alloc(&ow.Vimg, nc * p * vt) || !alloc(&ow.T, nc * p * tsz) ||
             !alloc(&ow.Vexp, nc * vt))
             return bail(fail(h, TQR_ERR_ALLOC, "tile storage allocation failed"));
+        if (nc && h->tree_L > 0 &&
+            (!alloc(&ow.Mimg, nc * h->dmax * vt) || !alloc(&ow.MT, nc * h->dmax * tsz) ||
+             !alloc64(&ow.Mt, h->dmax * tile)))
+            return bail(fail(h, TQR_ERR_ALLOC, "tree merge storage allocation failed"));
         if (nc && h->f32() &&
             (!alloc64(&ow.sc_col, p * tile) || !alloc64(&ow.sc_T, p * tsz) || !alloc64(&ow.sc_Vimg, p * tile) ||
              !alloc64(&ow.sc_Vexp, tile)))
@@ -480,7 +505,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
                 for (int j = k + 1; j < h->q; ++j) if (h->owner_of[j] == ow.id) { need_rb = true; break; }
         if (need_rb)
             for (int s = 0; s < 2; ++s)
-                if (!alloc(&ow.rb_tiles[s], p * vt) || !alloc(&ow.rb_T[s], p * tsz) || !alloc(&ow.rb_V[s], vt))
+                if (!alloc(&ow.rb_tiles[s], p * vt) || !alloc(&ow.rb_T[s], p * tsz) || !alloc(&ow.rb_V[s], vt) ||
+                    (h->tree_L > 0 && (!alloc(&ow.rb_M[s], h->dmax * vt) || !alloc(&ow.rb_MT[s], h->dmax * tsz))))
                     return bail(fail(h, TQR_ERR_ALLOC, "receive buffer allocation failed"));
         if (nc) {
             const size_t nfl = (size_t)p * (nb / ib) * 5;   // F + up to 4 sub-slice flags
@@ -555,30 +581,78 @@ cudaError_t from_tiles(const tqr_plan_s* h, void* dst, int64_t lda, int64_t gstr
     return tqr::launch_from_tiles<double>((double*)dst, lda, gstride, (const double*)src, cols, nc, colsz, h->nb,
                                           m_rows, n_valid, local_dst, s);
 }
-// Reflector data of panel k as seen by an update: images V (tile i at V + i*vt), T, explicit V.
+// Reflector data of panel k as seen by an update: images V (tile i at V + i*vt), T (tile i at
+// T + i*ib*nb), explicit V of the diagonal tile; tree mode: merge images / T (slot e).
 struct PanelRefs {
     void* V;
     void* T;
     void* Vexp;
+    void* M = nullptr;
+    void* MT = nullptr;
 };
-cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col_stride, int64_t tile_stride,
-                   int64_t ld, int group0, int gstride, int k, int w, int nslices, bool trans, cudaStream_t s) {
+// One update-kernel launch: reflector tiles k_head (UNMQR, if do_unmqr) and k_head+1..p_end-1
+// (TSMQR against row tile k_head) applied to nslices column slices of X.
+cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const void* Vexp, void* X, int64_t col_stride,
+                    int64_t tile_stride, int64_t ld, int group0, int gstride, int k_head, int p_end, int do_unmqr,
+                    int w, int nslices, bool trans, cudaStream_t s) {
     if (h->f32()) {
         tqr::UpdateArgsT<float> u;
-        u.V = (const float*)r.V; u.T = (const float*)r.T; u.Vexp = (const float*)r.Vexp; u.X = (float*)X;
+        u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
         u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
-        u.group0 = group0; u.gstride = gstride; u.k = k; u.p = h->p; u.do_unmqr = 1;
+        u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr;
         return tqr::launch_update_f32(h->nb, h->ib, w, u, nslices, trans, s);
     }
     tqr::UpdateArgs u;
-    u.V = (const double*)r.V; u.T = (const double*)r.T; u.Vexp = (const double*)r.Vexp; u.X = (double*)X;
+    u.V = (const double*)V; u.T = (const double*)T; u.Vexp = (const double*)Vexp; u.X = (double*)X;
     u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
-    u.group0 = group0; u.gstride = gstride; u.k = k; u.p = h->p; u.do_unmqr = 1;
+    u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr;
     return tqr::launch_update(h->nb, h->ib, w, u, nslices, trans, s);
+}
+// Q_k^T (trans) or Q_k applied to X.  Flat: one launch (UNMQR(k) + TSMQR(k+1..p-1)).  Tree (D > 1
+// domains of L tiles): per domain d, UNMQR of its head k + d*L and TSMQR of its tiles against the
+// head; then the merge chain TSMQR(head_e against head_0), e = 1..D-1 (row tiles k + e*L, i.e.
+// stride L*tile_stride).  Q is applied in the reverse order.  Returns the number of launches in *nl.
+cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col_stride, int64_t tile_stride,
+                   int64_t ld, int group0, int gstride, int k, int w, int nslices, bool trans, cudaStream_t s,
+                   int64_t* nl = nullptr) {
+    const int D = h->ndom(k), L = h->tree_L;
+    if (D == 1) {
+        if (nl) *nl += 1;
+        return update1(h, r.V, r.T, r.Vexp, X, col_stride, tile_stride, ld, group0, gstride, k, h->p, 1, w, nslices,
+                       trans, s);
+    }
+    auto dom = [&](int d) {
+        const int head = k + d * L, end = std::min(head + L, h->p);
+        const void* vex = d == 0 ? r.Vexp : h->at(r.V, (int64_t)head * h->vt);
+        return update1(h, r.V, r.T, vex, X, col_stride, tile_stride, ld, group0, gstride, head, end, 1, w, nslices,
+                       trans, s);
+    };
+    auto mrg = [&]() {
+        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L, ld, group0,
+                       gstride, 0, D, 0, w, nslices, trans, s);
+    };
+    if (nl) *nl += D + 1;
+    cudaError_t e = cudaSuccess;
+    if (trans) {
+        for (int d = 0; d < D && e == cudaSuccess; ++d) e = dom(d);
+        if (e == cudaSuccess) e = mrg();
+    } else {
+        e = mrg();
+        for (int d = D - 1; d >= 0 && e == cudaSuccess; --d) e = dom(d);
+    }
+    return e;
 }
 PanelRefs own_refs(const tqr_plan_s* h, Owner& O, int lc) {
     const int64_t p = h->p, tsz = (int64_t)h->ib * h->nb;
-    return {h->at(O.Vimg, lc * p * h->vt), h->at(O.T, lc * p * tsz), h->at(O.Vexp, lc * h->vt)};
+    PanelRefs r{h->at(O.Vimg, lc * p * h->vt), h->at(O.T, lc * p * tsz), h->at(O.Vexp, lc * h->vt)};
+    if (O.Mimg) {
+        r.M = h->at(O.Mimg, lc * h->dmax * h->vt);
+        r.MT = h->at(O.MT, lc * h->dmax * tsz);
+    }
+    return r;
+}
+PanelRefs recv_refs(const tqr_plan_s*, Owner& O, int slot) {
+    return {O.rb_tiles[slot], O.rb_T[slot], O.rb_V[slot], O.rb_M[slot], O.rb_MT[slot]};
 }
 }  // namespace
 
@@ -646,8 +720,29 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
         a.Vimg = h->at<double>(O.Vimg, lc * colsz);
         a.T = h->at<double>(O.T, lc * (int64_t)p * tsz);
         a.Vexp = h->at<double>(O.Vexp, lc * tile);
-        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O.s_panel));
-        h->launches++;
+        const int D = h->ndom(k);
+        if (D == 1) {
+            CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O.s_panel));
+            h->launches++;
+            return TQR_OK;
+        }
+        // tree: D TS domains (one CTA each), then the flat merge chain of the domain heads' R
+        // factors against head 0 (the panel kernel in TSQRT-only mode on the merge bottoms)
+        tqr::DomainArgs da{a.col, a.T, a.Vimg, a.Vexp, k, p, h->tree_L};
+        CUDA_TRY(h, tqr::launch_domains(nb, ib, da, D, O.s_panel));
+        CUDA_TRY(h, tqr::launch_merge_prep(nb, a.col, O.Mt, k, h->tree_L, D, O.s_panel));
+        const PanelRefs r = own_refs(h, O, lc);
+        tqr::PanelArgs m = a;
+        m.col = O.Mt;
+        m.T = (double*)r.MT;
+        m.Vimg = (double*)r.M;
+        m.Vexp = (double*)r.M;
+        m.k = 0;
+        m.p = D;
+        m.top = a.col + (int64_t)k * tile;
+        m.skip_ge = 1;
+        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m, O.s_panel));
+        h->launches += 3;
         return TQR_OK;
     }
     CUDA_TRY(h, tqr::launch_widen(h->at<float>(O.tiles, lc * colsz + k * tile), O.sc_col + k * tile,
@@ -708,7 +803,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 if (st) return st;
                 CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
             }
-            PanelRefs b = root ? own_refs(h, R, R.lidx[k]) : PanelRefs{R.rb_tiles[slot], R.rb_T[slot], R.rb_V[slot]};
+            PanelRefs b = root ? own_refs(h, R, R.lidx[k]) : recv_refs(h, R, slot);
             const ncclDataType_t dt = h->f32() ? ncclFloat32 : ncclFloat64;
             void* bv = h->at(b.V, k * vt);
             void* bt = h->at(b.T, k * tsz);
@@ -716,6 +811,11 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             NCCL_TRY(h, h->nccl->Broadcast(bv, bv, (size_t)(p - k) * vt, dt, ok, h->comm, R.s_comm));
             NCCL_TRY(h, h->nccl->Broadcast(bt, bt, (size_t)(p - k) * tsz, dt, ok, h->comm, R.s_comm));
             NCCL_TRY(h, h->nccl->Broadcast(b.Vexp, b.Vexp, (size_t)vt, dt, ok, h->comm, R.s_comm));
+            if (h->ndom(k) > 1) {
+                const size_t D = h->ndom(k);
+                NCCL_TRY(h, h->nccl->Broadcast(b.M, b.M, D * vt, dt, ok, h->comm, R.s_comm));
+                NCCL_TRY(h, h->nccl->Broadcast(b.MT, b.MT, D * tsz, dt, ok, h->comm, R.s_comm));
+            }
             NCCL_TRY(h, h->nccl->GroupEnd());
             CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
         } else {
@@ -739,6 +839,11 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_T[slot], k * tsz), D.dev, h->at(src.T, k * tsz), O->dev,
                                                 es * (size_t)(p - k) * tsz, D.s_comm));
                 CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, src.Vexp, O->dev, es * (size_t)vt, D.s_comm));
+                if (h->ndom(k) > 1) {
+                    const size_t nd = h->ndom(k);
+                    CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_M[slot], D.dev, src.M, O->dev, es * nd * vt, D.s_comm));
+                    CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_MT[slot], D.dev, src.MT, O->dev, es * nd * tsz, D.s_comm));
+                }
                 CUDA_TRY(h, cudaEventRecord(D.ev_recv[k], D.s_comm));
             }
         }
@@ -747,7 +852,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             CUDA_TRY(h, cudaSetDevice(D.dev));
             const bool mine = (D.id == ok);
             const int slot = k & 1;
-            const PanelRefs r = mine ? own_refs(h, D, D.lidx[k]) : PanelRefs{D.rb_tiles[slot], D.rb_T[slot], D.rb_V[slot]};
+            const PanelRefs r = mine ? own_refs(h, D, D.lidx[k]) : recv_refs(h, D, slot);
             cudaEvent_t ready = mine ? D.ev_panel[k] : D.ev_recv[k];
             // local columns j > k form a suffix [first, ncols) of D.cols
             int first = (int)(std::upper_bound(D.cols.begin(), D.cols.end(), k) - D.cols.begin());
@@ -758,8 +863,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, ready, 0));
                 if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_u[first % S][k - 1], 0));
                 const int wl = w_look(h);
-                CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, D.s_panel));
-                h->launches++;
+                CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, D.s_panel,
+                                   &h->launches));
                 first += 1;
             }
             CUDA_TRY(h, cudaEventRecord(D.ev_look[k], D.s_panel));
@@ -773,8 +878,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
                     if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[uu][k], su));
                     const int wb = w_bulk(h);
-                    CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, S, k, wb, ng * (nb / wb), true, su));
-                    h->launches++;
+                    CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, S, k, wb, ng * (nb / wb), true, su,
+                                       &h->launches));
                     if (h->profile) {
                         CUDA_TRY(h, cudaEventRecord(D.tm1[uu][k], su));
                         D.tm_used[uu][k] = 1;
@@ -873,8 +978,7 @@ static tqr_status apply_device(tqr_plan h, char trans, void* Bw, int64_t ldw, in
         const int k = fwd ? s_ : q - 1 - s_;
         Owner* O = h->local(h->owner_of[k]);
         const PanelRefs r = own_refs(h, *O, O->lidx[k]);
-        CUDA_TRY(h, update(h, r, Bw, (int64_t)nb * ldw, nb, ldw, 0, 1, k, 32, (int)nslices, fwd, s));
-        h->launches++;
+        CUDA_TRY(h, update(h, r, Bw, (int64_t)nb * ldw, nb, ldw, 0, 1, k, 32, (int)nslices, fwd, s, &h->launches));
     }
     return TQR_OK;
 }

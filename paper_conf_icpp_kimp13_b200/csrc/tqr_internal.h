@@ -16,7 +16,24 @@ struct PanelArgs {
     unsigned epoch;    // value published for this launch (monotone across launches)
     int k;             // step (tile column / diagonal tile row)
     int p;             // number of row tiles
+    double* top = nullptr;   // TS "top" tile override (null: col + k*nb*nb)
+    int skip_ge = 0;         // 1: tile k is already triangular (a merge chain): TSQRT tiles k+1..p-1 only
 };
+
+// TS-domain step (NEXT-1 tree; paper's TT elimination P:L409-419): one CTA per domain
+// [k + d*L, min(k + (d+1)*L, p)) of panel column k: GEQRT of the domain head, then TSQRT of the
+// domain's other tiles against it.  Head d's explicit V image goes to Vexp (d = 0) or to the
+// head tile's own image slot (d > 0); its T to the head tile's T slot.
+struct DomainArgs {
+    double* col;
+    double* T;
+    double* Vimg;
+    double* Vexp;
+    int k, p, L;
+};
+cudaError_t launch_domains(int nb, int ib, const DomainArgs& a, int ndom, cudaStream_t s);
+// merge inputs: Mt[e] = triu(tile k + e*L) (zeros below the diagonal), e = 1..ndom-1
+cudaError_t launch_merge_prep(int nb, const double* col, double* Mt, int k, int L, int ndom, cudaStream_t s);
 
 // Trailing update of step k over `ngroups` column groups (UNMQR + TSMQR chain), or the
 // application of panel k's Q^T / Q to a right-hand side block (tqr_apply_qt).  T = element type.

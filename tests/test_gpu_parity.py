@@ -383,3 +383,47 @@ def test_full_size_c4_tall_skinny():
     assert orth <= 4.0 * orth_ref and orth <= 2.5e-13
     del Ad, Rd, E, Q2
     torch.cuda.empty_cache()
+
+
+TREES = [
+    # (m, n, nb, ib, L): TS domains of L tiles + flat TT merge chain (NEXT-1), forced
+    (512, 128, 64, 16, 2),      # p=8, q=2: 4 domains at step 0, 4 at step 1 (last domain 1 tile)
+    (1024, 256, 64, 16, 3),     # p=16, q=4: uneven domains, 6 -> 5 domains
+    (2048, 512, 128, 32, 4),    # p=16, q=4 at nb=128
+    (3072, 512, 512, 32, 2),    # q=1 at nb=512: 3 domains
+    (1000, 300, 64, 16, 3),     # ragged both ways
+    (768, 768, 256, 32, 1),     # L=1: every tile its own domain (pure TT-merge chain)
+]
+
+
+@pytest.mark.parametrize("m,n,nb,ib,L", TREES)
+def test_tree_matches_oracle(m, n, nb, ib, L):
+    A = synthetic.gaussian(m, n, 5000 + m + n + nb + L)
+    plan, Rg = gpu_qr(A, nb, ib, tree_domain=L)
+    ref = oracle.qr(A)
+    assert colnorm_rel_err(np.triu(Rg[:n]), ref.R) <= R_TOL
+    assert np.all(np.tril(Rg, -1) == 0.0)
+    Q, res = thin_q_and_residual(plan, A, Rg)
+    assert res <= RES_TOL, res
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0))
+    B = synthetic.gaussian(m, 2, 5100 + m)
+    Bd = dev_colmajor(B)
+    plan.solve_ls(Bd)
+    np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
+    plan.close()
+
+
+def test_tree_auto_for_single_column_and_partition():
+    """q == 1 picks the tree automatically; guide-array partitions with logical devices replay the
+    same tree through the broadcast path (merge images / T travel with the panel)."""
+    m, n, nb, ib = 8192, 512, 512, 32           # p = 16 -> L = 2, 8 domains
+    A = synthetic.gaussian(m, n, 5200)
+    plan, Rg = gpu_qr(A, nb, ib)
+    assert colnorm_rel_err(np.triu(Rg[:n]), oracle.qr(A).R) <= R_TOL
+    _, Rf = gpu_qr(A, nb, ib, tree_domain=-1)
+    assert colnorm_rel_err(np.triu(Rg[:n]), np.triu(Rf[:n])) <= R_TOL
+    m2, n2 = 1024, 512
+    A2 = synthetic.gaussian(m2, n2, 5201)
+    _, R1 = gpu_qr(A2, 64, 16, tree_domain=3)
+    _, R2 = gpu_qr(A2, 64, 16, tree_domain=3, ndev=3, guide=[2, 0, 1], logical_devices=True)
+    assert np.array_equal(R1, R2)
