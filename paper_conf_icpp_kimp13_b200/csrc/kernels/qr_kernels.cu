@@ -186,6 +186,7 @@ __global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
     const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
     unsigned vph = 0;
     stage_init(sf);
+    TQR_PP0();
     for (int i = head; i < end; ++i) {
         double* Ai = a.col + (int64_t)i * tile;
         double* Ti = a.T + (int64_t)i * IB * NB;
@@ -210,6 +211,7 @@ __global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
                                                                     vph);
             }
             __syncthreads();   // top rows written by the applies -> Rsm reads below
+            TQR_PP(4);
             if (ge) {
                 factor_block<NB, IB, true>(X, sf, b * IB);
             } else {
@@ -220,6 +222,7 @@ __global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
                 __syncthreads();
                 factor_block<NB, IB, false>(X, sf, b * IB);
             }
+            TQR_PP(5);
             X.store(Ai + (int64_t)b * IB * NB, NB);
 #pragma unroll
             for (int mf = 0; mf < IB / 8; ++mf) {
@@ -250,6 +253,7 @@ __global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
             }
             __threadfence_block();
             __syncthreads();
+            TQR_PP(6);
         }
     }
 }

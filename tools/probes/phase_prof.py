@@ -31,6 +31,10 @@ pt = sum(buf[16 + i] for i in range(4))
 if pt:
     print("panel last-leader chain:", ", ".join("%s %.1f%%" % (nm, 100.0 * buf[16 + i] / pt) for i, nm in
           enumerate(["flag waits", "applies", "gather+factor", "publish"])), "total Mcycles %.1f" % (pt / 1e6))
+dt = sum(buf[20 + i] for i in range(3))
+if dt:
+    print("domain kernel (last CTA):", ", ".join("%s %.1f%%" % (nm, 100.0 * buf[20 + i] / dt) for i, nm in
+          enumerate(["applies", "factor", "store+image+T"])), "total Mcycles %.1f" % (dt / 1e6))
 ft = sum(buf[24 + i] for i in range(3))
 if ft:
     print("factor_block (last CTA): columns %.1f Mcyc, Gram %.1f Mcyc, dlarft recurrence %.1f Mcyc" %
