@@ -190,6 +190,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-lookahead", action="store_true")
+    ap.add_argument("--tree", type=int, default=0,
+                    help="elimination tree: 0 auto (tree for q == 1), -1 flat TS, L > 0 TS domains of L tiles")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -224,7 +226,7 @@ def main():
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
     plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, rank=rank, world=world, nccl_id=nccl_id,
-                    lookahead=not args.no_lookahead, profile=True)
+                    lookahead=not args.no_lookahead, profile=True, tree_domain=args.tree)
 
     def step(Ain, Aout):
         plan.load(Ain)
@@ -335,6 +337,7 @@ def main():
             "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
                        "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": list(range(world)),
                        "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
+                       "tree": args.tree,
                        "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (es * m * n / 2 ** 30)
                        if es * m * n > L2_BYTES else "input fits L2 (no flush)"},
             "roofline": roofline,

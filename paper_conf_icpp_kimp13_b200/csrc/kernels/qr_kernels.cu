@@ -58,11 +58,17 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     using G = Geom<NB, IB, IB>;
     constexpr int NBLK = NB / IB;
     constexpr int S = IB / W;
-    const int b = blockIdx.x / (S + 1), u = blockIdx.x % (S + 1);
+    // multi-job launch (tree mode): job = domain [head, end) of the panel column, its own wavefront
+    const int job = blockIdx.x / (NBLK * (S + 1));
+    const int cta = blockIdx.x % (NBLK * (S + 1));
+    const int b = cta / (S + 1), u = cta % (S + 1);
     const bool leader = (u == S);              // the factor CTA of block b
     const int64_t tile = (int64_t)NB * NB;
+    const int head = a.L > 0 ? a.k + job * a.L : a.k;
+    const int end = a.L > 0 ? min(head + a.L, a.p) : a.p;
     double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
-    double* Akk = a.top ? a.top : col + (int64_t)a.k * tile;
+    double* Akk = a.top ? a.top : col + (int64_t)head * tile;
+    double* Vexp = (head == a.k) ? a.Vexp : a.Vimg + (int64_t)head * tile;
     unsigned* F = a.flags;                                   // p * NBLK
     unsigned* Gf = a.flags + (int64_t)a.p * NBLK;            // p * NBLK * S
     const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
@@ -70,10 +76,10 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     stage_init(sa);
     TQR_PP0();
 
-    for (int i = a.k + a.skip_ge; i < a.p; ++i) {
+    for (int i = head + a.skip_ge; i < end; ++i) {
         double* Ai = col + (int64_t)i * tile;
         double* Ti = a.T + (int64_t)i * IB * NB;
-        const bool ge = (i == a.k);
+        const bool ge = (i == head);
         const int c0 = b * IB + u * W;         // first column of this sub-slice
         if (!leader && b > 0) {
             Slice<NB, W, IB> X;
@@ -83,7 +89,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
                 TQR_PP(1);
                 flag_wait_geq(F + (int64_t)i * NBLK + bp, a.epoch);
                 TQR_PP(0);
-                const double* Vb = (ge ? a.Vexp : a.Vimg + (int64_t)i * tile) + (int64_t)bp * IB * NB;
+                const double* Vb = (ge ? Vexp : a.Vimg + (int64_t)i * tile) + (int64_t)bp * IB * NB;
                 if (lane_id() == 0) fence_proxy_async_global();   // sibling CTA's generic stores -> bulk copy
                 stage_first(sa, Vb);
                 if (ge)
@@ -129,7 +135,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         // GEQRT: rows < b*IB of these columns are R rows finished by the sub-slice applies and may
         // already be updated as TS "tops" of tile k+1 by the sub-slice CTAs: store rows >= b*IB only.
         Xf.store_rows_from(Ai + (int64_t)b * IB * NB, NB, ge ? b * IB : 0);
-        double* img = ge ? a.Vexp : a.Vimg + (int64_t)i * tile;
+        double* img = ge ? Vexp : a.Vimg + (int64_t)i * tile;
 #pragma unroll
         for (int mf = 0; mf < IB / 8; ++mf) {
             const int cb = mf * 8 + g;                 // column within the block
@@ -416,12 +422,12 @@ __global__ void zero_diag_check_kernel(const T* __restrict__ R, int64_t ldr, int
 
 // ============================================================================ launchers
 template <int NB, int IB, int W>
-static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s) {
+static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s, int njobs) {
     const size_t smem = std::max(sizeof(Smem<NB, IB, IB, true>), sizeof(Smem<NB, W, IB, true>));
     auto kern = panel_kernel<NB, IB, W>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    kern<<<(NB / IB) * (IB / W + 1), kThreads, smem, s>>>(a);
+    kern<<<njobs * (NB / IB) * (IB / W + 1), kThreads, smem, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -448,18 +454,18 @@ static cudaError_t launch_update_t(const UpdateArgs& a, int nslices, bool trans,
     if (nb == NB_ && ib == IB_) { return CALL; }
 
 template <int NB, int IB, int W>
-static cudaError_t launch_panel_chk(const PanelArgs& a, cudaStream_t s) {
-    if constexpr (W >= 8) return launch_panel_t<NB, IB, W>(a, s);
+static cudaError_t launch_panel_chk(const PanelArgs& a, cudaStream_t s, int njobs) {
+    if constexpr (W >= 8) return launch_panel_t<NB, IB, W>(a, s, njobs);
     else return cudaErrorInvalidValue;
 }
 
 // split: sub-slices per ib column block (1, 2 or 4; W = ib / split >= 8)
-cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s) {
+cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s, int njobs) {
 #define TQR_PAN(NB_, IB_)                                                          \
     if (nb == NB_ && ib == IB_) {                                                  \
-        if (split == 1) return launch_panel_chk<NB_, IB_, IB_>(a, s);             \
-        if (split == 2) return launch_panel_chk<NB_, IB_, IB_ / 2>(a, s);         \
-        if (split == 4) return launch_panel_chk<NB_, IB_, IB_ / 4>(a, s);         \
+        if (split == 1) return launch_panel_chk<NB_, IB_, IB_>(a, s, njobs);      \
+        if (split == 2) return launch_panel_chk<NB_, IB_, IB_ / 2>(a, s, njobs);  \
+        if (split == 4) return launch_panel_chk<NB_, IB_, IB_ / 4>(a, s, njobs);  \
         return cudaErrorInvalidValue;                                              \
     }
     TQR_PAN(64, 16) TQR_PAN(64, 32) TQR_PAN(128, 16) TQR_PAN(128, 32)

@@ -99,6 +99,8 @@ struct tqr_plan_s {
     int tree_L = 0;                 // TS-domain length (tiles); 0 = flat TS chain
     int dmax = 1;                   // max domains of any step = ceil(p / tree_L)
     int ndom(int k) const { return tree_L > 0 ? (p - k + tree_L - 1) / tree_L : 1; }
+    bool tree_one_cta = true;       // domain phase: one CTA per domain (long domains) or wavefront jobs
+    int tree_split = 1;             // panel split of the wavefront domain jobs
     std::vector<Owner> owners;      // in-process: ndev entries; multi-process: 1 (this rank)
     const tqr::NcclApi* nccl = nullptr;
     ncclComm_t comm = nullptr;
@@ -421,6 +423,20 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         h->tree_L = std::max(2, (h->p + sms - 1) / sms);
     }
     if (h->tree_L >= h->p) h->tree_L = 0;
+    // Domain phase: a single CTA per domain pays ~2 ms per nb = 512 tile but runs one domain per
+    // SM -- right for many long domains (C4); a few short domains run faster as wavefront jobs.
+    if (h->tree_L > 0) {
+        int sms = 148;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+        h->tree_one_cta = h->ndom(0) * 2 > sms;
+        if (const char* e = getenv("TQR_TREE_ONE_CTA")) h->tree_one_cta = atoi(e) != 0;
+        const int nblk = nb / ib;
+        const int D0 = h->ndom(0);
+        h->tree_split = (D0 * nblk * 5 <= sms) ? 4 : (D0 * nblk * 3 <= sms ? 2 : 1);
+        if (ib < 32 && h->tree_split > 2) h->tree_split = 2;
+        if (ib / h->tree_split < 8) h->tree_split = 1;
+        if (const char* e = getenv("TQR_TREE_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->tree_split = v; }
+    }
     if (h->tree_L > 0 && dtype != TQR_F64) { h->tree_L = 0; if (o.tree_domain > 0) { delete h; return fail(nullptr, TQR_ERR_UNSUPPORTED, "tree mode: FP64 only in this build"); } }
     h->dmax = h->ndom(0);
     // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
@@ -728,8 +744,15 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
         }
         // tree: D TS domains (one CTA each), then the flat merge chain of the domain heads' R
         // factors against head 0 (the panel kernel in TSQRT-only mode on the merge bottoms)
-        tqr::DomainArgs da{a.col, a.T, a.Vimg, a.Vexp, k, p, h->tree_L};
-        CUDA_TRY(h, tqr::launch_domains(nb, ib, da, D, O.s_panel));
+        if (h->tree_one_cta) {
+            tqr::DomainArgs da{a.col, a.T, a.Vimg, a.Vexp, k, p, h->tree_L};
+            CUDA_TRY(h, tqr::launch_domains(nb, ib, da, D, O.s_panel));
+        } else {
+            // short domains: each domain its own wavefront (the panel kernel, one job per domain)
+            tqr::PanelArgs dj = a;
+            dj.L = h->tree_L;
+            CUDA_TRY(h, tqr::launch_panel(nb, ib, h->tree_split, dj, O.s_panel, D));
+        }
         CUDA_TRY(h, tqr::launch_merge_prep(nb, a.col, O.Mt, k, h->tree_L, D, O.s_panel));
         const PanelRefs r = own_refs(h, O, lc);
         tqr::PanelArgs m = a;

@@ -18,6 +18,8 @@ struct PanelArgs {
     int p;             // number of row tiles
     double* top = nullptr;   // TS "top" tile override (null: col + k*nb*nb)
     int skip_ge = 0;         // 1: tile k is already triangular (a merge chain): TSQRT tiles k+1..p-1 only
+    int L = 0;               // > 0: multi-job (tree mode) -- job d = domain [k + d*L, min(k + (d+1)*L, p)),
+                             //      head d's explicit V image in Vexp (d = 0) or Vimg slot k + d*L
 };
 
 // TS-domain step (NEXT-1 tree; paper's TT elimination P:L409-419): one CTA per domain
@@ -55,7 +57,7 @@ struct UpdateArgsT {
 using UpdateArgs = UpdateArgsT<double>;
 
 // split = apply CTAs per ib column block (1, 2, 4): grid = (nb/ib) * (split + 1)
-cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s);
+cudaError_t launch_panel(int nb, int ib, int split, const PanelArgs& a, cudaStream_t s, int njobs = 1);
 // nslices CTAs; CTA b works on columns [b*w, b*w + w) counted from group0 (groups are nb wide)
 cudaError_t launch_update(int nb, int ib, int w, const UpdateArgs& a, int nslices, bool trans, cudaStream_t s);
 // a1: src column group of local column lc at src + (local_src ? lc : cols[lc])*src_group_stride

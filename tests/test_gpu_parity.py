@@ -396,8 +396,12 @@ TREES = [
 ]
 
 
+@pytest.mark.parametrize("one_cta", ["0", "1"])
 @pytest.mark.parametrize("m,n,nb,ib,L", TREES)
-def test_tree_matches_oracle(m, n, nb, ib, L):
+def test_tree_matches_oracle(m, n, nb, ib, L, one_cta, monkeypatch):
+    """Both domain phases: wavefront jobs (panel kernel, one job per domain) and one CTA per
+    domain (domain_kernel)."""
+    monkeypatch.setenv("TQR_TREE_ONE_CTA", one_cta)
     A = synthetic.gaussian(m, n, 5000 + m + n + nb + L)
     plan, Rg = gpu_qr(A, nb, ib, tree_domain=L)
     ref = oracle.qr(A)
