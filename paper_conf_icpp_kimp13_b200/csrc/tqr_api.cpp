@@ -52,7 +52,9 @@ struct Owner {
     void* rb_tiles[2] = {nullptr, nullptr};
     void* rb_T[2] = {nullptr, nullptr};
     void* rb_V[2] = {nullptr, nullptr};
-    unsigned* flags = nullptr;      // p * (nb/ib)
+    unsigned* flags = nullptr;      // p * (nb/ib) * 5 panel-kernel publication flags
+    unsigned* mflags = nullptr;     // tree mode: the merge chain's own flags (the domain jobs of the
+                                    // same step stamp the main flags with the same epoch)
     void* io = nullptr;             // m x (nb*ncols) column-major mirror for host / remote I/O
     // tree mode (TS domains + flat TT merge chain, NEXT-1): per owned column, Dmax merge slots
     void* Mimg = nullptr;           // ncols * Dmax * vt   stage images of the merge reflectors (slot e)
@@ -87,6 +89,9 @@ struct tqr_plan_s {
     int nb = 0, ib = 0, p = 0, q = 0;
     tqr_dtype dtype = TQR_F64;
     int es = 8;                     // element size in bytes
+    bool f32_tc = false;            // FP32 update on 3xTF32 tensor cores (experimental, TQR_F32_KERNEL=tf32:
+                                    // same speed as the FFMA kernel so far and ~3x the orthogonality
+                                    // error, above the FP32 bar at n >= 256); default SIMT FFMA
     int64_t vt = 0;                 // elements of one reflector-tile stage image (F64: nb*nb)
     int ndev = 1;
     std::vector<int32_t> guide;
@@ -166,7 +171,7 @@ bool supported_nb_ib(int nb, int ib) {
 
 // Slice width of the bulk update kernel and of the (latency-critical) lookahead column.
 int w_bulk(const tqr_plan_s*) { return 32; }
-int w_look(const tqr_plan_s* h) { return h->nb >= 256 ? 8 : 16; }
+int w_look(const tqr_plan_s* h) { return (h->nb >= 256 && !(h->f32() && h->f32_tc)) ? 8 : 16; }
 
 double flops_update(const tqr_plan_s* h, int k, int ncols) {
     const double nb3 = (double)h->nb * h->nb * h->nb;
@@ -180,7 +185,7 @@ double flops_panel(const tqr_plan_s* h, int k) {
 void free_owner(Owner& o) {
     cudaSetDevice(o.dev);
     auto F = [](void* p) { if (p) cudaFree(p); };
-    F(o.cols_dev); F(o.tiles); F(o.Vimg); F(o.T); F(o.Vexp); F(o.flags); F(o.io);
+    F(o.cols_dev); F(o.tiles); F(o.Vimg); F(o.T); F(o.Vexp); F(o.flags); F(o.mflags); F(o.io);
     F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp); F(o.Mimg); F(o.MT); F(o.Mt);
     for (int s = 0; s < 2; ++s) { F(o.rb_M[s]); F(o.rb_MT[s]); }
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
@@ -406,7 +411,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)((m + nb - 1) / nb); h->q = (int)((n + nb - 1) / nb);
     h->dtype = dtype; h->ndev = ndev; h->guide = g;
     h->es = (dtype == TQR_F32) ? 4 : 8;
-    h->vt = (dtype == TQR_F32) ? tqr::f32_img_tile(nb, ib) : (int64_t)nb * nb;
+    if (const char* e = getenv("TQR_F32_KERNEL")) h->f32_tc = strcmp(e, "tf32") == 0;
+    h->vt = (dtype == TQR_F32) ? (h->f32_tc ? tqr::tf32_img_tile(nb) : tqr::f32_img_tile(nb, ib)) : (int64_t)nb * nb;
     h->logical = o.logical_devices != 0;
     h->rank = use_nccl ? o.rank : 0;
     h->world = world;
@@ -529,6 +535,9 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
             if (cudaMalloc(&ow.flags, nfl * sizeof(unsigned)) != cudaSuccess ||
                 cudaMemset(ow.flags, 0, nfl * sizeof(unsigned)) != cudaSuccess)
                 return bail(fail(h, TQR_ERR_ALLOC, "flag allocation failed"));
+            if (h->tree_L > 0 && (cudaMalloc(&ow.mflags, nfl * sizeof(unsigned)) != cudaSuccess ||
+                                  cudaMemset(ow.mflags, 0, nfl * sizeof(unsigned)) != cudaSuccess))
+                return bail(fail(h, TQR_ERR_ALLOC, "flag allocation failed"));
         }
     }
     // peer access between physical owners (single-process, several GPUs)
@@ -616,6 +625,7 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
         u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
         u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
         u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr;
+        if (h->f32_tc) return tqr::launch_update_tf32(h->nb, h->ib, w, u, nslices, trans, s);
         return tqr::launch_update_f32(h->nb, h->ib, w, u, nslices, trans, s);
     }
     tqr::UpdateArgs u;
@@ -764,6 +774,7 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
         m.p = D;
         m.top = a.col + (int64_t)k * tile;
         m.skip_ge = 1;
+        m.flags = O.mflags;
         CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m, O.s_panel));
         h->launches += 3;
         return TQR_OK;
@@ -773,8 +784,12 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
     a.col = O.sc_col; a.Vimg = O.sc_Vimg; a.T = O.sc_T; a.Vexp = O.sc_Vexp;
     CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O.s_panel));
     const PanelRefs r = own_refs(h, O, lc);
-    CUDA_TRY(h, tqr::launch_narrow_panel(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz), (float*)r.T,
-                                         (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
+    if (h->f32_tc)
+        CUDA_TRY(h, tqr::launch_narrow_panel_tf32(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz),
+                                                  (float*)r.T, (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
+    else
+        CUDA_TRY(h, tqr::launch_narrow_panel(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz), (float*)r.T,
+                                             (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
     h->launches += 3;
     return TQR_OK;
 }
