@@ -95,6 +95,10 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
                 if (ge)
                     apply_block<NB, W, IB, true, true, true, true>(X, sa, Vb, Ti + (int64_t)bp * IB * IB, nullptr,
                                                                    0, bp * IB, nullptr, vph);
+                else if (a.skip_ge)   // TT merge: bottom triangular, rows >= (bp+1)*IB of V and X are zero
+                    apply_block<NB, W, IB, true, true, true, true>(X, sa, Vb, Ti + (int64_t)bp * IB * IB,
+                                                                   Akk + (int64_t)c0 * NB + bp * IB, NB, 0,
+                                                                   nullptr, vph, (bp + 1) * IB);
                 else
                     apply_block<NB, W, IB, true, true, true, false>(X, sa, Vb, Ti + (int64_t)bp * IB * IB,
                                                                     Akk + (int64_t)c0 * NB + bp * IB, NB, 0,

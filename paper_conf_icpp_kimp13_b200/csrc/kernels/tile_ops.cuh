@@ -193,13 +193,14 @@ __device__ __forceinline__ void stage_first(Smem<NB, W, IB, FACT>& sm, const dou
 //   Ts   : T block s (IB x IB column-major, ld = IB) = T_tile + s*IB*IB (zeros below diagonal).
 //   top  : if non-null, the X1 rows (IB x W, element (r, c) at top[c*ldtop + r]).
 //   next : stage image of the following call's block -- its half A is staged here -- or null.
-//   KM   : kmin may be > 0 (UNMQR / GEQRT blocks); false compiles the TS path branch-free.
+//   KM   : kmin may be > 0 (UNMQR / GEQRT blocks) or kmax < NB (TT merges: a triangular bottom
+//          keeps V and X zero on rows >= kmax); false compiles the TS path branch-free.
 template <int NB, int W, int IB, bool FACT, bool TRANS, bool CG, bool KM>
 __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB, FACT>& sm,
                                             const double* __restrict__ Vs,
                                             const double* __restrict__ Ts,
                                             double* top, int64_t ldtop, int kmin,
-                                            const double* next, unsigned& vph) {
+                                            const double* next, unsigned& vph, int kmax = 1 << 30) {
     using G = Geom<NB, W, IB>;
     using SM = Smem<NB, W, IB, FACT>;
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
@@ -239,7 +240,7 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
             for (int j = 0; j < G::JC; ++j) c1[h][mf][j][0] = c1[h][mf][j][1] = 0.0;
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
-            if (KM && rbase + nf * 8 + 8 <= kmin) continue;  // V rows all zero (warp-uniform)
+            if (KM && (rbase + nf * 8 + 8 <= kmin || rbase + nf * 8 >= kmax)) continue;  // V rows all zero (warp-uniform)
             double2 b[G::JC];
 #pragma unroll
             for (int j = 0; j < G::JC; ++j)
@@ -355,7 +356,7 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
             for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + h * G::HC + kk + t];
 #pragma unroll
             for (int nf = 0; nf < G::NF; ++nf) {
-                if (KM && rbase + nf * 8 + 8 <= kmin) continue;
+                if (KM && (rbase + nf * 8 + 8 <= kmin || rbase + nf * 8 >= kmax)) continue;
                 const double b = vh[vst_off<NB, W, IB>(nf * 8 + g, kk + t)];
 #pragma unroll
                 for (int mf = 0; mf < G::MF; ++mf) dmma(X.acc[mf][nf][0], X.acc[mf][nf][1], a[mf], b);
