@@ -11,7 +11,6 @@
 #include <algorithm>
 #include <cstdio>
 #include "tile_ops_f32.cuh"
-#include "tile_ops_tf32.cuh"
 #include "../tqr_internal.h"
 
 namespace tqr {
@@ -148,159 +147,7 @@ TQR_FITS32(256, 16) TQR_FITS32(256, 32) TQR_FITS32(512, 16) TQR_FITS32(512, 32)
 
 }  // namespace f32
 
-namespace tf32 {
 
-// Same chain / block order as f32::update_kernel32, on 3xTF32 mma.sync (tile_ops_tf32.cuh).
-template <int NB, int W, int IB, bool TRANS>
-__global__ void __launch_bounds__(kThreads, 1) update_kernel_tf32(UpdateArgsT<float> a) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    auto& sm = *reinterpret_cast<Smem<NB, W, IB>*>(smem_raw);
-    constexpr int SPG = NB / W;
-    constexpr int NBLK = NB / IB;
-    constexpr int64_t VT = img_tile<NB, IB>();
-    const int grp = blockIdx.x / SPG;
-    const int c0 = (blockIdx.x % SPG) * W;
-    float* Xg = a.X + (int64_t)(a.group0 + grp * a.gstride) * a.col_stride + (int64_t)c0 * a.ld;
-    float* Xk = Xg + (int64_t)a.k * a.tile_stride;
-    Slice<NB, W, IB> X;
-    stage_init(sm);
-    unsigned vph = 0;
-    const int ntiles = a.p - a.k - 1 + (a.do_unmqr ? 1 : 0);
-    auto tile_of = [&](int q) -> int {
-        if (TRANS) return a.do_unmqr ? (q == 0 ? -1 : a.k + q) : a.k + 1 + q;
-        return (q < a.p - a.k - 1) ? a.p - 1 - q : -1;
-    };
-    auto vblock = [&](int ti, int s) -> const float* {
-        return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * VT) + (int64_t)s * NB * IB * 2;
-    };
-    auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
-    if (ntiles > 0) stage(sm, vblock(tile_of(0), blk(0)), 0);
-    for (int q = 0; q < ntiles; ++q) {
-        const int ti = tile_of(q);
-        float* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
-        const float* Tt = a.T + (int64_t)(ti < 0 ? a.k : ti) * IB * NB;
-        X.load(Xi, a.ld);
-        for (int si = 0; si < NBLK; ++si) {
-            const int s = blk(si);
-            const float* nxt = nullptr;
-            if (si + 1 < NBLK) nxt = vblock(ti, blk(si + 1));
-            else if (q + 1 < ntiles) nxt = vblock(tile_of(q + 1), blk(0));
-            apply_block<NB, W, IB, TRANS>(X, sm, vblock(ti, s), Tt + (int64_t)s * IB * IB,
-                                          ti < 0 ? nullptr : Xk + s * IB, a.ld, ti < 0 ? s * IB : 0, nxt, vph);
-        }
-        X.store(Xi, a.ld);
-        __syncthreads();
-    }
-}
-
-// Panel out for the 3xTF32 update: as f32::narrow_panel_kernel, writing the hi/lo 8x8-block
-// stage image (img_off) from a shared-memory copy of the FP32-rounded chunk.
-template <int NB, int IB>
-__global__ void __launch_bounds__(256) narrow_panel_tf32_kernel(const double* __restrict__ sc, const double* __restrict__ T64,
-                                                               float* __restrict__ tiles, float* __restrict__ T32,
-                                                               float* __restrict__ Vimg, float* __restrict__ Vexp, int k) {
-    using G = Geom<NB, 16, IB>;
-    constexpr int RC = NB < 128 ? NB : 128;       // rows per CTA (a multiple of RW)
-    __shared__ float st[RC][IB + 1];
-    const int nch = NB / RC;
-    const int chunk = blockIdx.x % nch, s = (blockIdx.x / nch) % (NB / IB), i = k + blockIdx.x / (nch * (NB / IB));
-    const int64_t tile = (int64_t)NB * NB;
-    const bool ge = (i == k);
-    const double* src = sc + (int64_t)i * tile;
-    float* dt = tiles + (int64_t)i * tile;
-    const int r0 = chunk * RC;
-    for (int e = threadIdx.x; e < IB * RC; e += blockDim.x) {
-        const int kk = e / RC, rl = e % RC;
-        const int c = s * IB + kk, r = r0 + rl;
-        const double v = src[(int64_t)c * NB + r];
-        dt[(int64_t)c * NB + r] = (float)v;
-        st[rl][kk] = ge ? (r > c ? (float)v : (r == c ? 1.f : 0.f)) : (float)v;
-    }
-    __syncthreads();
-    // contiguous image region of rows r0 .. r0 + RC - 1 of block s: RC/RW warp ranges x 2 halves
-    float* img = (ge ? Vexp : Vimg + (int64_t)i * img_tile<NB, IB>()) + (int64_t)s * NB * IB * 2 +
-                 (int64_t)r0 * IB * 2;
-    for (int e = threadIdx.x; e < RC * IB * 2; e += blockDim.x) {
-        const int q = e / (G::RW * IB * 2), rem = e % (G::RW * IB * 2);
-        const int h = rem / G::HALF, rb = rem % G::HALF;
-        const int blkid = rb >> 7, idx = rb & 127;
-        const int nf = blkid / G::JH, jj = blkid % G::JH;
-        const int c8 = idx >> 4, hl = idx & 1;
-        const int r8 = ((((idx >> 3) & 1) ^ ((c8 >> 1) & 1)) << 2) | (((idx >> 2) & 1) << 1) | ((idx >> 1) & 1);
-        const int rl = q * G::RW + nf * 8 + r8, kk = h * G::HC + jj * 8 + c8;
-        const float f = st[rl][kk];
-        const float hi = __uint_as_float(tf32_round(f));
-        img[e] = (hl == 0) ? hi : __uint_as_float(tf32_round(f - hi));
-    }
-    if (chunk == 0) {
-        const double* ts = T64 + (int64_t)i * IB * NB + (int64_t)s * IB * IB;
-        float* td = T32 + (int64_t)i * IB * NB + (int64_t)s * IB * IB;
-        for (int e = threadIdx.x; e < IB * IB; e += blockDim.x) td[e] = (float)ts[e];
-    }
-}
-
-template <int NB, int W, int IB>
-static cudaError_t launch_update_t(const UpdateArgsT<float>& a, int nslices, bool trans, cudaStream_t s) {
-  if constexpr (W % 16 != 0) {
-    return cudaErrorInvalidValue;
-  } else {
-    const size_t smem = sizeof(Smem<NB, W, IB>);
-    if (nslices <= 0) return cudaSuccess;
-    if (trans) {
-        auto kern = update_kernel_tf32<NB, W, IB, true>;
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        kern<<<nslices, kThreads, smem, s>>>(a);
-    } else {
-        auto kern = update_kernel_tf32<NB, W, IB, false>;
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        kern<<<nslices, kThreads, smem, s>>>(a);
-    }
-    return cudaGetLastError();
-  }
-}
-#define TQR_FITSTF(NB_, IB_)                                                                  \
-    static_assert(sizeof(Smem<NB_, 16, IB_>) <= f32::kMaxSmem, "tf32 update smem W=16");     \
-    static_assert(sizeof(Smem<NB_, 32, IB_>) <= f32::kMaxSmem, "tf32 update smem W=32");
-TQR_FITSTF(64, 16) TQR_FITSTF(64, 32) TQR_FITSTF(128, 16) TQR_FITSTF(128, 32)
-TQR_FITSTF(256, 16) TQR_FITSTF(256, 32) TQR_FITSTF(512, 16) TQR_FITSTF(512, 32)
-#undef TQR_FITSTF
-
-}  // namespace tf32
-
-// w: 16 or 32 (m16 fragments)
-cudaError_t launch_update_tf32(int nb, int ib, int w, const UpdateArgsT<float>& a, int nslices, bool trans,
-                               cudaStream_t s) {
-#define TQR_UPDTF(NB_, IB_)                                                                   \
-    if (nb == NB_ && ib == IB_) {                                                             \
-        if (w == 16) return tf32::launch_update_t<NB_, 16, IB_>(a, nslices, trans, s);        \
-        if (w == 32) return tf32::launch_update_t<NB_, 32, IB_>(a, nslices, trans, s);        \
-        return cudaErrorInvalidValue;                                                         \
-    }
-    TQR_UPDTF(64, 16) TQR_UPDTF(64, 32) TQR_UPDTF(128, 16) TQR_UPDTF(128, 32)
-    TQR_UPDTF(256, 16) TQR_UPDTF(256, 32) TQR_UPDTF(512, 16) TQR_UPDTF(512, 32)
-#undef TQR_UPDTF
-    return cudaErrorInvalidValue;
-}
-
-cudaError_t launch_narrow_panel_tf32(int nb, int ib, const double* sc, const double* T64, float* tiles, float* T32,
-                                     float* Vimg, float* Vexp, int k, int p, cudaStream_t s) {
-    const int ntiles = p - k;
-    if (ntiles <= 0) return cudaSuccess;
-#define TQR_NART(NB_, IB_)                                                                                    \
-    if (nb == NB_ && ib == IB_) {                                                                             \
-        const int grid = ntiles * (NB_ / IB_) * (NB_ >= 128 ? NB_ / 128 : 1);                                 \
-        tf32::narrow_panel_tf32_kernel<NB_, IB_><<<grid, 256, 0, s>>>(sc, T64, tiles, T32, Vimg, Vexp, k);    \
-        return cudaGetLastError();                                                                            \
-    }
-    TQR_NART(64, 16) TQR_NART(64, 32) TQR_NART(128, 16) TQR_NART(128, 32)
-    TQR_NART(256, 16) TQR_NART(256, 32) TQR_NART(512, 16) TQR_NART(512, 32)
-#undef TQR_NART
-    return cudaErrorInvalidValue;
-}
-
-int64_t tf32_img_tile(int nb) { return (int64_t)nb * nb * 2; }
 
 cudaError_t launch_update_f32(int nb, int ib, int w, const UpdateArgsT<float>& a, int nslices, bool trans,
                               cudaStream_t s) {

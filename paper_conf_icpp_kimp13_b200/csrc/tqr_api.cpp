@@ -89,9 +89,6 @@ struct tqr_plan_s {
     int nb = 0, ib = 0, p = 0, q = 0;
     tqr_dtype dtype = TQR_F64;
     int es = 8;                     // element size in bytes
-    bool f32_tc = false;            // FP32 update on 3xTF32 tensor cores (experimental, TQR_F32_KERNEL=tf32:
-                                    // same speed as the FFMA kernel so far and ~3x the orthogonality
-                                    // error, above the FP32 bar at n >= 256); default SIMT FFMA
     int64_t vt = 0;                 // elements of one reflector-tile stage image (F64: nb*nb)
     int ndev = 1;
     std::vector<int32_t> guide;
@@ -171,7 +168,7 @@ bool supported_nb_ib(int nb, int ib) {
 
 // Slice width of the bulk update kernel and of the (latency-critical) lookahead column.
 int w_bulk(const tqr_plan_s*) { return 32; }
-int w_look(const tqr_plan_s* h) { return (h->nb >= 256 && !(h->f32() && h->f32_tc)) ? 8 : 16; }
+int w_look(const tqr_plan_s* h) { return h->nb >= 256 ? 8 : 16; }
 
 double flops_update(const tqr_plan_s* h, int k, int ncols) {
     const double nb3 = (double)h->nb * h->nb * h->nb;
@@ -411,8 +408,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)((m + nb - 1) / nb); h->q = (int)((n + nb - 1) / nb);
     h->dtype = dtype; h->ndev = ndev; h->guide = g;
     h->es = (dtype == TQR_F32) ? 4 : 8;
-    if (const char* e = getenv("TQR_F32_KERNEL")) h->f32_tc = strcmp(e, "tf32") == 0;
-    h->vt = (dtype == TQR_F32) ? (h->f32_tc ? tqr::tf32_img_tile(nb) : tqr::f32_img_tile(nb, ib)) : (int64_t)nb * nb;
+    h->vt = (dtype == TQR_F32) ? tqr::f32_img_tile(nb, ib) : (int64_t)nb * nb;
     h->logical = o.logical_devices != 0;
     h->rank = use_nccl ? o.rank : 0;
     h->world = world;
@@ -625,7 +621,6 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
         u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
         u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
         u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr;
-        if (h->f32_tc) return tqr::launch_update_tf32(h->nb, h->ib, w, u, nslices, trans, s);
         return tqr::launch_update_f32(h->nb, h->ib, w, u, nslices, trans, s);
     }
     tqr::UpdateArgs u;
@@ -784,12 +779,8 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
     a.col = O.sc_col; a.Vimg = O.sc_Vimg; a.T = O.sc_T; a.Vexp = O.sc_Vexp;
     CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, a, O.s_panel));
     const PanelRefs r = own_refs(h, O, lc);
-    if (h->f32_tc)
-        CUDA_TRY(h, tqr::launch_narrow_panel_tf32(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz),
-                                                  (float*)r.T, (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
-    else
-        CUDA_TRY(h, tqr::launch_narrow_panel(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz), (float*)r.T,
-                                             (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
+    CUDA_TRY(h, tqr::launch_narrow_panel(nb, ib, O.sc_col, O.sc_T, h->at<float>(O.tiles, lc * colsz), (float*)r.T,
+                                         (float*)r.V, (float*)r.Vexp, k, p, O.s_panel));
     h->launches += 3;
     return TQR_OK;
 }

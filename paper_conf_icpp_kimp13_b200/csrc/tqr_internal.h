@@ -88,13 +88,6 @@ cudaError_t launch_widen(const float* src, double* dst, int64_t n, cudaStream_t 
 cudaError_t launch_narrow_panel(int nb, int ib, const double* sc, const double* T64, float* tiles, float* T32,
                                 float* Vimg, float* Vexp, int k, int p, cudaStream_t s);
 int64_t f32_img_tile(int nb, int ib);
-// 3xTF32 tensor-core update (mma.sync m16n8k8 TF32, hi/lo split); V / Vexp are hi/lo stage images
-// (tf32_img_tile elements per tile); w in {16, 32}
-cudaError_t launch_update_tf32(int nb, int ib, int w, const UpdateArgsT<float>& a, int nslices, bool trans,
-                               cudaStream_t s);
-cudaError_t launch_narrow_panel_tf32(int nb, int ib, const double* sc, const double* T64, float* tiles, float* T32,
-                                     float* Vimg, float* Vexp, int k, int p, cudaStream_t s);
-int64_t tf32_img_tile(int nb);
 size_t panel_smem_bytes(int nb, int ib);
 size_t update_smem_bytes(int nb, int ib, int w);
 
