@@ -192,6 +192,8 @@ def main():
     ap.add_argument("--no-lookahead", action="store_true")
     ap.add_argument("--tree", type=int, default=0,
                     help="elimination tree: 0 auto (tree for q == 1), -1 flat TS, L > 0 TS domains of L tiles")
+    ap.add_argument("--tree-group", type=int, default=0,
+                    help="tree merge: 0 auto (two-level for >= 16 domains), -1 flat chain, G > 1 groups of G")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -226,7 +228,8 @@ def main():
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
     plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, rank=rank, world=world, nccl_id=nccl_id,
-                    lookahead=not args.no_lookahead, profile=True, tree_domain=args.tree)
+                    lookahead=not args.no_lookahead, profile=True, tree_domain=args.tree,
+                    tree_group=args.tree_group)
 
     def step(Ain, Aout):
         plan.load(Ain)
@@ -271,29 +274,35 @@ def main():
     value = fl / (ms * 1e-3) / 1e9
     peak, peak_src = fp32_peak_tflops() if f32 else fp64_peak_tflops()
 
-    # ---- e2e: pinned host in, pinned host out, copies inside the timed region
+    # ---- e2e: the public call a user makes, tqr_factor on a pinned host A (in place: A <- R).
+    # The library pipelines the host->device column loads and the device->host R stores with the
+    # factorization; both copies are inside the timed region.  A is restored from the pristine
+    # copy between iterations (untimed).
     e2e = None
     if not args.no_e2e:
         Ah = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
         Ah.copy_(A0)
-        Rh = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
-        step(Ah, Rh)
+        plan.factor(Ah)
         torch.cuda.synchronize()
-        barrier()
-        t0 = time.perf_counter()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
         ke = max(1, min(K, 2))
+        tot = 0.0
         for _ in range(ke):
-            step(Ah, Rh)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        ems = max_over_ranks(e0.elapsed_time(e1) / ke)
+            Ah.copy_(A0)
+            torch.cuda.synchronize()
+            barrier()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            plan.factor(Ah)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            tot += e0.elapsed_time(e1)
+        ems = max_over_ranks(tot / ke)
         e2e = {"value": round(fl / (ems * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
                "ms_per_step": round(ems, 3), "h2d_bytes_per_step": es * m * n, "d2h_bytes_per_step": es * m * n,
-               "api": "tqr_load(host) + tqr_factor_tiles + tqr_store_r(host) == tqr_factor on pinned host A"}
-        del Ah, Rh
+               "api": "tqr_factor(pinned host A): per-column H2D + layout convert, factorization and per-column "
+                      "R-out + D2H overlapped inside the call"}
+        del Ah
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -337,7 +346,7 @@ def main():
             "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
                        "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": list(range(world)),
                        "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
-                       "tree": args.tree,
+                       "tree": args.tree, "tree_group": args.tree_group,
                        "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (es * m * n / 2 ** 30)
                        if es * m * n > L2_BYTES else "input fits L2 (no flush)"},
             "roofline": roofline,

@@ -72,6 +72,12 @@ typedef struct {
      * and tqr_apply_qt replay the same tree.  0 = auto (tree for a single column tile, q == 1,
      * with L = ceil(p / SM count)), -1 = always flat TS, L > 0 = domains of L tiles (FP64 only). */
     int32_t tree_domain;
+    /* Tree mode: how the D domain heads are merged.  0 = auto (two-level when D >= 16, groups of
+     * ceil(sqrt(D))), -1 = one flat TT chain of D - 1 merges, G > 1 = two-level: the heads of each
+     * group of G consecutive domains are merged into the group's first head by concurrent TT
+     * chains, then the group heads into head 0 by one chain (G - 1 + ceil(D/G) - 1 sequential
+     * merges instead of D - 1). */
+    int32_t tree_group;
 } tqr_options;
 
 /*

@@ -66,20 +66,25 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
     const int64_t tile = (int64_t)NB * NB;
     const int head = a.L > 0 ? a.k + job * a.L : a.k;
     const int end = a.L > 0 ? min(head + a.L, a.p) : a.p;
-    double* col = a.col;                       // tiles of panel column k: tile i at col + i*tile
-    double* Akk = a.top ? a.top : col + (int64_t)head * tile;
+    double* col = a.col;                       // tiles of panel column k: tile i at col + i*stride*tile
+    const int st = a.stride;
+    double* Akk = (a.top && job == 0) ? a.top : col + (int64_t)head * st * tile;
     double* Vexp = (head == a.k) ? a.Vexp : a.Vimg + (int64_t)head * tile;
     unsigned* F = a.flags;                                   // p * NBLK
-    unsigned* Gf = a.flags + (int64_t)a.p * NBLK;            // p * NBLK * S
+    // G(slot, b, u) at Gf + (slot*NBLK + b)*4 + u: independent of S, so launches of one epoch with
+    // different splits (the two merge levels) never alias each other's flags
+    unsigned* Gf = a.flags + (int64_t)(a.fslots > 0 ? a.fslots : a.p) * NBLK;
+    static_assert(S <= 4, "G flag stride");
     const int g = lane_id() >> 2, t = lane_id() & 3, wq = warp_id();
     unsigned vph = 0;
     stage_init(sa);
     TQR_PP0();
 
-    for (int i = head + a.skip_ge; i < end; ++i) {
+    for (int ic = head + a.skip_ge; ic < end; ++ic) {
+        const int i = ic * st;                 // slot of chain index ic
         double* Ai = col + (int64_t)i * tile;
         double* Ti = a.T + (int64_t)i * IB * NB;
-        const bool ge = (i == head);
+        const bool ge = (ic == head);
         const int c0 = b * IB + u * W;         // first column of this sub-slice
         if (!leader && b > 0) {
             Slice<NB, W, IB> X;
@@ -110,7 +115,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
             if (b > 0) {
                 __threadfence();
                 __syncthreads();
-                if (threadIdx.x == 0) flag_release(Gf + ((int64_t)i * NBLK + b) * S + u, a.epoch);
+                if (threadIdx.x == 0) flag_release(Gf + ((int64_t)i * NBLK + b) * 4 + u, a.epoch);
                 TQR_TRACE("cta %d (b%d u%d) tile %d published G\n", blockIdx.x, b, u, i);
             }
             continue;
@@ -118,7 +123,7 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         // ---- leader: gather the IB columns of block b and factor them
         TQR_TRACE("cta %d (b%d u%d) tile %d leader waits G\n", blockIdx.x, b, u, i);
         if (b > 0)
-            for (int up = 0; up < S; ++up) flag_wait_geq(Gf + ((int64_t)i * NBLK + b) * S + up, a.epoch);
+            for (int up = 0; up < S; ++up) flag_wait_geq(Gf + ((int64_t)i * NBLK + b) * 4 + up, a.epoch);
         TQR_TRACE("cta %d (b%d u%d) tile %d leader factors\n", blockIdx.x, b, u, i);
         TQR_PP(0);
         Slice<NB, IB, IB> Xf;
@@ -308,14 +313,14 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
         return (q < a.p - a.k - 1) ? a.p - 1 - q : -1;
     };
     auto vblock = [&](int ti, int s) -> const double* {
-        return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * vtile) + (int64_t)s * IB * NB;
+        return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;
     };
     auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
     if (ntiles > 0) stage_first(sm, vblock(tile_of(0), blk(0)));
     for (int q = 0; q < ntiles; ++q) {
         const int ti = tile_of(q);
         double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
-        const double* Tt = a.T + (int64_t)(ti < 0 ? a.k : ti) * IB * NB;
+        const double* Tt = a.T + (int64_t)(ti < 0 ? a.k : ti * a.vstride) * IB * NB;
         X.load(Xi, a.ld);
         for (int si = 0; si < NBLK; ++si) {
             const int s = blk(si);

@@ -21,6 +21,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -68,6 +69,8 @@ struct Owner {
     double* sc_Vimg = nullptr;      // p * nb*nb
     double* sc_Vexp = nullptr;      // nb*nb
     cudaStream_t s_panel = nullptr, s_upd = nullptr, s_comm = nullptr;
+    cudaStream_t s_io = nullptr;                    // streamed tqr_factor: per-column H2D + a1, a8 + D2H
+    std::vector<cudaEvent_t> ev_load;               // ev_load[lc]: local column lc resident in tile layout
     std::vector<cudaStream_t> s_u;                  // bulk-update streams (column lc -> s_u[lc % S])
     std::vector<cudaEvent_t> ev_panel, ev_recv, ev_look;
     std::vector<std::vector<cudaEvent_t>> ev_u;     // ev_u[u][k]: stream u finished its step-k updates
@@ -100,6 +103,15 @@ struct tqr_plan_s {
     int panel_split = 1;            // sub-slice CTAs per ib column block in the panel kernel
     int tree_L = 0;                 // TS-domain length (tiles); 0 = flat TS chain
     int dmax = 1;                   // max domains of any step = ceil(p / tree_L)
+    int tree_G = 0;                 // two-level merge: groups of G domains (0 = one flat merge chain)
+    int merge_split = 1;            // panel sub-slice split of the level-1 merge jobs
+    // streamed tqr_factor (caller A not on the owner's device): column loads overlap the
+    // factorization (panel k / the step-0 update of column j wait for ev_load), R of column k is
+    // written back on s_io as soon as PANEL(k) completes
+    bool streamed = false;
+    void* sA = nullptr;
+    int64_t slda = 0;
+    int ngroups(int D) const { return (tree_G > 1 && D > tree_G) ? (D + tree_G - 1) / tree_G : 1; }
     int ndom(int k) const { return tree_L > 0 ? (p - k + tree_L - 1) / tree_L : 1; }
     bool tree_one_cta = true;       // domain phase: one CTA per domain (long domains) or wavefront jobs
     int tree_split = 1;             // panel split of the wavefront domain jobs
@@ -186,7 +198,7 @@ void free_owner(Owner& o) {
     F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp); F(o.Mimg); F(o.MT); F(o.Mt);
     for (int s = 0; s < 2; ++s) { F(o.rb_M[s]); F(o.rb_MT[s]); }
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
-    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref})
+    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref, &o.ev_load})
         for (auto e : *v) if (e) cudaEventDestroy(e);
     for (auto* vv : {&o.ev_u, &o.tm0, &o.tm1})
         for (auto& v : *vv) for (auto e : v) if (e) cudaEventDestroy(e);
@@ -194,6 +206,7 @@ void free_owner(Owner& o) {
     if (o.s_panel) cudaStreamDestroy(o.s_panel);
     if (o.s_upd) cudaStreamDestroy(o.s_upd);
     if (o.s_comm) cudaStreamDestroy(o.s_comm);
+    if (o.s_io) cudaStreamDestroy(o.s_io);
 }
 
 // Host-side DAG (Fig. 3) per rank, the same order the executor issues.
@@ -271,6 +284,7 @@ tqr_status sync_all(tqr_plan h) {
         CUDA_TRY(h, cudaStreamSynchronize(o.s_upd));
         CUDA_TRY(h, cudaStreamSynchronize(o.s_comm));
         for (auto su : o.s_u) CUDA_TRY(h, cudaStreamSynchronize(su));
+        if (o.s_io) CUDA_TRY(h, cudaStreamSynchronize(o.s_io));
     }
     return TQR_OK;
 }
@@ -441,6 +455,18 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     }
     if (h->tree_L > 0 && dtype != TQR_F64) { h->tree_L = 0; if (o.tree_domain > 0) { delete h; return fail(nullptr, TQR_ERR_UNSUPPORTED, "tree mode: FP64 only in this build"); } }
     h->dmax = h->ndom(0);
+    // Two-level merge of the D domain heads: groups of G ~ sqrt(D) merged concurrently, then the
+    // group heads (D - 1 sequential merges -> G - 1 + ceil(D/G) - 1).
+    if (h->tree_L > 0) {
+        const int D0 = h->dmax;
+        if (o.tree_group > 1) h->tree_G = o.tree_group;
+        else if (o.tree_group == 0 && D0 >= 16) h->tree_G = (int)std::ceil(std::sqrt((double)D0));
+        if (const char* e = getenv("TQR_TREE_GROUP")) h->tree_G = atoi(e);
+        if (h->tree_G < 2) h->tree_G = 0;
+        h->merge_split = (ib >= 32) ? 2 : 1;
+        if (const char* e = getenv("TQR_MERGE_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->merge_split = v; }
+        if (ib / h->merge_split < 8) h->merge_split = 1;
+    }
     // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
     // panel is on the critical path (few trailing columns per panel step or several owners).
     h->panel_split = (h->q <= 4) ? 4 : 2;   // measured: 4 for tall / few columns, 2 otherwise
@@ -467,7 +493,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
             if (h->owner_of[j] == ow.id) { ow.lidx[j] = (int32_t)ow.cols.size(); ow.cols.push_back(j); }
         if (cudaSetDevice(ow.dev) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "cudaSetDevice(%d)", ow.dev));
         auto mk = [&](cudaStream_t* s, int prio) { return cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, prio); };
-        if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi))
+        if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi) || mk(&ow.s_io, prio_hi))
             return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
         const int S = h->nstreams;
         ow.s_u.assign(S, nullptr);
@@ -480,7 +506,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
                     return false;
             return true;
         };
-        bool ok = mkev(ow.ev_panel, h->q, false) && mkev(ow.ev_recv, h->q, false) && mkev(ow.ev_look, h->q, false);
+        bool ok = mkev(ow.ev_panel, h->q, false) && mkev(ow.ev_recv, h->q, false) && mkev(ow.ev_look, h->q, false) &&
+                  mkev(ow.ev_load, (int)ow.cols.size(), false);
         ow.ev_u.resize(S);
         for (int u = 0; u < S && ok; ++u) ok = mkev(ow.ev_u[u], h->q, false);
         if (ok && h->profile) {
@@ -615,7 +642,7 @@ struct PanelRefs {
 // (TSMQR against row tile k_head) applied to nslices column slices of X.
 cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const void* Vexp, void* X, int64_t col_stride,
                     int64_t tile_stride, int64_t ld, int group0, int gstride, int k_head, int p_end, int do_unmqr,
-                    int w, int nslices, bool trans, cudaStream_t s) {
+                    int w, int nslices, bool trans, cudaStream_t s, int vstride = 1) {
     if (h->f32()) {
         tqr::UpdateArgsT<float> u;
         u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
@@ -626,13 +653,16 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
     tqr::UpdateArgs u;
     u.V = (const double*)V; u.T = (const double*)T; u.Vexp = (const double*)Vexp; u.X = (double*)X;
     u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
-    u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr;
+    u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr; u.vstride = vstride;
     return tqr::launch_update(h->nb, h->ib, w, u, nslices, trans, s);
 }
 // Q_k^T (trans) or Q_k applied to X.  Flat: one launch (UNMQR(k) + TSMQR(k+1..p-1)).  Tree (D > 1
 // domains of L tiles): per domain d, UNMQR of its head k + d*L and TSMQR of its tiles against the
 // head; then the merge chain TSMQR(head_e against head_0), e = 1..D-1 (row tiles k + e*L, i.e.
-// stride L*tile_stride).  Q is applied in the reverse order.  Returns the number of launches in *nl.
+// stride L*tile_stride) -- or, with groups of G domains (two-level merge), per group g the chain
+// of heads gG+1..gG+G-1 against head gG, then the chain of group heads G, 2G, .. against head 0
+// (merge slot e holds the reflectors of the merge whose bottom was head e).  Q is applied in the
+// reverse order.  Returns the number of launches in *nl.
 cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col_stride, int64_t tile_stride,
                    int64_t ld, int group0, int gstride, int k, int w, int nslices, bool trans, cudaStream_t s,
                    int64_t* nl = nullptr) {
@@ -648,17 +678,40 @@ cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col
         return update1(h, r.V, r.T, vex, X, col_stride, tile_stride, ld, group0, gstride, head, end, 1, w, nslices,
                        trans, s);
     };
-    auto mrg = [&]() {
+    const int NG = h->ngroups(D), G = h->tree_G;
+    const int64_t tsz = (int64_t)h->ib * h->nb;
+    auto mrg = [&]() {   // flat merge chain
         return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L, ld, group0,
                        gstride, 0, D, 0, w, nslices, trans, s);
     };
-    if (nl) *nl += D + 1;
+    auto grp = [&](int g) {   // level 1: group g's chain against its head gG
+        const int h0 = g * G, len = std::min(G, D - h0);
+        if (len < 2) return cudaSuccess;
+        return update1(h, h->at(r.M, (int64_t)h0 * h->vt), h->at(r.MT, (int64_t)h0 * tsz), r.M,
+                       h->at(X, (int64_t)(k + h0 * L) * tile_stride), col_stride, tile_stride * L, ld, group0, gstride,
+                       0, len, 0, w, nslices, trans, s);
+    };
+    auto top = [&]() {   // level 2: group heads G, 2G, .. against head 0 (merge slots stride G)
+        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L * G, ld,
+                       group0, gstride, 0, NG, 0, w, nslices, trans, s, G);
+    };
+    if (nl) *nl += D + (NG > 1 ? NG + 1 : 1);
     cudaError_t e = cudaSuccess;
     if (trans) {
         for (int d = 0; d < D && e == cudaSuccess; ++d) e = dom(d);
-        if (e == cudaSuccess) e = mrg();
+        if (NG == 1) {
+            if (e == cudaSuccess) e = mrg();
+        } else {
+            for (int g = 0; g < NG && e == cudaSuccess; ++g) e = grp(g);
+            if (e == cudaSuccess) e = top();
+        }
     } else {
-        e = mrg();
+        if (NG == 1) {
+            e = mrg();
+        } else {
+            e = top();
+            for (int g = NG - 1; g >= 0 && e == cudaSuccess; --g) e = grp(g);
+        }
         for (int d = D - 1; d >= 0 && e == cudaSuccess; --d) e = dom(d);
     }
     return e;
@@ -770,8 +823,23 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
         m.top = a.col + (int64_t)k * tile;
         m.skip_ge = 1;
         m.flags = O.mflags;
-        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m, O.s_panel));
-        h->launches += 3;
+        m.fslots = p;
+        const int NG = h->ngroups(D);
+        if (NG == 1) {
+            CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m, O.s_panel));
+            h->launches += 3;
+            return TQR_OK;
+        }
+        // two-level merge: NG concurrent chains (job g merges heads gG+1.. into head gG; job 0's
+        // top is the real head tile, job g > 0's is merge slot gG), then the chain of group heads
+        tqr::PanelArgs m1 = m;
+        m1.L = h->tree_G;
+        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->merge_split, m1, O.s_panel, NG));
+        tqr::PanelArgs m2 = m;
+        m2.stride = h->tree_G;
+        m2.p = NG;
+        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m2, O.s_panel));
+        h->launches += 4;
         return TQR_OK;
     }
     CUDA_TRY(h, tqr::launch_widen(h->at<float>(O.tiles, lc * colsz + k * tile), O.sc_col + k * tile,
@@ -814,11 +882,26 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
         if (O) {
             CUDA_TRY(h, cudaSetDevice(O->dev));
             if (k > 0 && !h->lookahead) { tqr_status st = wait_all_u(*O, O->s_panel, k - 1); if (st) return st; }
+            if (h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(O->s_panel, O->ev_load[O->lidx[k]], 0));
             if (h->profile) CUDA_TRY(h, cudaEventRecord(O->tp0[k], O->s_panel));
             tqr_status st = launch_panel_step(h, *O, k, epoch0 + (unsigned)k + 1);
             if (st) return st;
             if (h->profile) { CUDA_TRY(h, cudaEventRecord(O->tp1[k], O->s_panel)); O->tp_used[k] = 1; }
             CUDA_TRY(h, cudaEventRecord(O->ev_panel[k], O->s_panel));
+            if (h->streamed) {
+                // column k is final once PANEL(k) is done (later steps touch columns > k only, and
+                // updates read the reflectors from the stage images): a8 + D2H on the I/O stream
+                const int lc = O->lidx[k];
+                const size_t es = h->es;
+                void* slab = h->at(O->io, (int64_t)lc * h->m * nb);
+                CUDA_TRY(h, cudaStreamWaitEvent(O->s_io, O->ev_panel[k], 0));
+                CUDA_TRY(h, from_tiles(h, slab, h->m, h->m * nb, h->at(O->tiles, lc * colsz), O->cols_dev + lc, 1,
+                                       h->m, h->n, 1, O->s_io));
+                CUDA_TRY(h, cudaMemcpy2DAsync(static_cast<char*>(h->sA) + (int64_t)k * nb * h->slda * es,
+                                              h->slda * es, slab, h->m * es, h->m * es, group_cols(h, k),
+                                              cudaMemcpyDefault, O->s_io));
+                h->launches++;
+            }
         }
         // ---- BCAST(k): the reflector-tile images k..p-1, their T factors and the explicit V
         if (h->multiproc()) {
@@ -891,6 +974,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 // lookahead: column k+1 first, on the high-priority panel stream
                 CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, ready, 0));
                 if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_u[first % S][k - 1], 0));
+                if (k == 0 && h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_load[first], 0));
                 const int wl = w_look(h);
                 CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, D.s_panel,
                                    &h->launches));
@@ -907,8 +991,17 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
                     if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[uu][k], su));
                     const int wb = w_bulk(h);
-                    CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, S, k, wb, ng * (nb / wb), true, su,
-                                       &h->launches));
+                    if (k == 0 && h->streamed) {
+                        // step 0 of a streamed factor: one launch per column, each after its load
+                        for (int c = g0; c < nloc; c += S) {
+                            CUDA_TRY(h, cudaStreamWaitEvent(su, D.ev_load[c], 0));
+                            CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, c, S, k, wb, nb / wb, true, su,
+                                               &h->launches));
+                        }
+                    } else {
+                        CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, S, k, wb, ng * (nb / wb), true, su,
+                                           &h->launches));
+                    }
                     if (h->profile) {
                         CUDA_TRY(h, cudaEventRecord(D.tm1[uu][k], su));
                         D.tm_used[uu][k] = 1;
@@ -982,12 +1075,52 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
     return sync_all(h);
 }
 
+// A not resident on the owners' devices (host memory, or another GPU): the I/O is pipelined with
+// the factorization -- column tile j is copied in and converted (a1) on the owner's I/O stream,
+// PANEL(j) and the step-0 update of column j wait only for column j, and R of column k (a8) is
+// copied out as soon as PANEL(k) completes, so only the first column's load and the last
+// column's store are exposed.  A is in place (the columns being read are never the ones written).
 tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
-    tqr_status st = tqr_load(h, A, lda);
-    if (st) return st;
-    st = tqr_factor_tiles(h);
-    if (st) return st;
-    return tqr_store_r(h, A, lda);
+    if (!h) return TQR_ERR_ARG;
+    if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "factor: A is NULL or lda < m");
+    const PtrInfo pi = classify(A);
+    bool resident = true;
+    for (auto& o : h->owners)
+        if (!o.cols.empty() && !(pi.kind == Mem::Device && pi.dev == o.dev)) resident = false;
+    if (resident || getenv("TQR_NO_STREAMED_IO")) {
+        tqr_status st = tqr_load(h, A, lda);
+        if (st) return st;
+        st = tqr_factor_tiles(h);
+        if (st) return st;
+        return tqr_store_r(h, A, lda);
+    }
+    const int64_t nb = h->nb, es = h->es, colsz = (int64_t)h->p * nb * nb;
+    h->factored = false;
+    { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
+    for (auto& o : h->owners) {
+        if (o.cols.empty()) continue;
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        tqr_status st = ensure_io(h, o);
+        if (st) return st;
+        for (int lc = 0; lc < (int)o.cols.size(); ++lc) {
+            const int64_t j = o.cols[lc];
+            void* slab = h->at(o.io, (int64_t)lc * h->m * nb);
+            CUDA_TRY(h, cudaMemcpy2DAsync(slab, h->m * es, static_cast<const char*>(A) + j * nb * lda * es, lda * es,
+                                          h->m * es, group_cols(h, j), cudaMemcpyDefault, o.s_io));
+            CUDA_TRY(h, to_tiles(h, slab, h->m, h->m * nb, h->at(o.tiles, lc * colsz), o.cols_dev + lc, 1, 1, o.s_io));
+            CUDA_TRY(h, cudaEventRecord(o.ev_load[lc], o.s_io));
+            h->launches++;
+        }
+    }
+    h->streamed = true;
+    h->sA = A;
+    h->slda = lda;
+    tqr_status st = tqr_factor_tiles(h);
+    h->streamed = false;
+    h->sA = nullptr;
+    if (st) sync_all(h);
+    return st;
 }
 
 // ------------------------------------------------------------------ apply Q^T / Q, solve

@@ -19,7 +19,12 @@ struct PanelArgs {
     double* top = nullptr;   // TS "top" tile override (null: col + k*nb*nb)
     int skip_ge = 0;         // 1: tile k is already triangular (a merge chain): TSQRT tiles k+1..p-1 only
     int L = 0;               // > 0: multi-job (tree mode) -- job d = domain [k + d*L, min(k + (d+1)*L, p)),
-                             //      head d's explicit V image in Vexp (d = 0) or Vimg slot k + d*L
+                             //      head d's explicit V image in Vexp (d = 0) or Vimg slot k + d*L;
+                             //      with skip_ge (merge groups) the top override applies to job 0 only,
+                             //      job d > 0 merges into its own head slot
+    int fslots = 0;          // > 0: slot rows of the F flag block (G flags follow it); 0 = p
+    int stride = 1;          // chain index i addresses slot i*stride of col / T / Vimg / flags (the
+                             //      second level of a two-level merge walks the group heads)
 };
 
 // TS-domain step (NEXT-1 tree; paper's TT elimination P:L409-419): one CTA per domain
@@ -53,6 +58,7 @@ struct UpdateArgsT {
     int gstride;         // group index step between consecutive groups of this launch
     int k, p;
     int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
+    int vstride = 1;     // reflector tile i at V + i*vstride*image tile, T + i*vstride*ib*nb
 };
 using UpdateArgs = UpdateArgsT<double>;
 

@@ -178,6 +178,29 @@ def test_host_pointer_and_pinned_paths_match_device():
     assert np.array_equal(np.triu(Ap.numpy()[:n]), np.triu(Rd[:n]))
 
 
+@pytest.mark.parametrize("m,n,nb,ib,kw", [
+    (1024, 768, 128, 32, {}),                                              # q = 6
+    (1000, 700, 128, 32, {"ndev": 3, "guide": [2, 0, 1], "logical_devices": True}),   # ragged, 3 owners
+    (4096, 256, 256, 32, {"tree_domain": 2}),                              # tree + two-level merge
+    (512, 512, 64, 16, {"lookahead": False}),
+])
+def test_streamed_host_factor_bitwise(m, n, nb, ib, kw, monkeypatch):
+    """tqr_factor on a host A pipelines the column loads / R stores with the factorization (panel k
+    and the step-0 update of column j wait only for their own column); the arithmetic is the
+    device-resident path's, so A <- R must agree bitwise, including the zeroed lower part."""
+    A = synthetic.gaussian(m, n, 90 + m + n)
+    _, Rd = gpu_qr(A, nb, ib, **kw)
+    plan = tqr.Plan(m, n, nb, ib, **kw)
+    Ap = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    plan.factor(Ap)
+    assert np.array_equal(Ap.numpy(), Rd)
+    monkeypatch.setenv("TQR_NO_STREAMED_IO", "1")          # the three-phase path on the same plan
+    Ap2 = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    plan.factor(Ap2)
+    assert np.array_equal(Ap2.numpy(), Rd)
+    plan.close()
+
+
 @pytest.mark.parametrize("ndev,guide", [(2, None), (2, [1, 0]), (3, [1, 0, 1, 0, 1, 2]), (4, [0, 0, 1, 3, 2])])
 def test_logical_devices_partition_bitwise(ndev, guide):
     """Guide-array partitions (Eq. 12) on logical devices: identical R to the 1-owner run."""
@@ -415,6 +438,40 @@ def test_tree_matches_oracle(m, n, nb, ib, L, one_cta, monkeypatch):
     plan.solve_ls(Bd)
     np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
     plan.close()
+
+
+MERGES = [
+    # (m, n, nb, ib, L, G): two-level merge -- groups of G domain heads, then the group heads
+    (1024, 128, 64, 16, 1, 4),      # p=16: 16 domains -> 4 groups of 4 (step 1: 15 -> 4, last of 3)
+    (2048, 256, 64, 16, 2, 3),      # p=32, q=4: 16 -> 6 groups (last of 1 domain), ragged per step
+    (1000, 300, 64, 16, 1, 5),      # ragged both ways
+    (8192, 512, 512, 32, 2, 3),     # q=1 at nb=512: 8 domains -> groups 3,3,2
+    (8192, 512, 512, 32, 1, 4),     # 16 domains -> 4 x 4
+]
+
+
+@pytest.mark.parametrize("m,n,nb,ib,L,G", MERGES)
+def test_two_level_merge_matches_oracle(m, n, nb, ib, L, G):
+    A = synthetic.gaussian(m, n, 5300 + m + n + nb + L + G)
+    plan, Rg = gpu_qr(A, nb, ib, tree_domain=L, tree_group=G)
+    ref = oracle.qr(A)
+    assert colnorm_rel_err(np.triu(Rg[:n]), ref.R) <= R_TOL
+    assert np.all(np.tril(Rg, -1) == 0.0)
+    Q, res = thin_q_and_residual(plan, A, Rg)
+    assert res <= RES_TOL, res
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0))
+    B = synthetic.gaussian(m, 2, 5400 + m)
+    Bd = dev_colmajor(B)
+    plan.solve_ls(Bd)
+    np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
+    plan.close()
+    # the flat merge chain reaches the same R (unique) and the logical-device partition replays
+    # the two-level tree through the broadcast path bitwise
+    _, Rf = gpu_qr(A, nb, ib, tree_domain=L, tree_group=-1)
+    assert colnorm_rel_err(np.triu(Rg[:n]), np.triu(Rf[:n])) <= R_TOL
+    if n > nb:
+        _, Rp = gpu_qr(A, nb, ib, tree_domain=L, tree_group=G, ndev=2, guide=[1, 0], logical_devices=True)
+        assert np.array_equal(Rg, Rp)
 
 
 def test_tree_auto_for_single_column_and_partition():
