@@ -316,7 +316,16 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
         return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;
     };
     auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
-    if (ntiles > 0) stage_first(sm, vblock(tile_of(0), blk(0)));
+    auto wait_tile = [&](int ti) {   // lookahead overlapped with the panel: tile ti published?
+        if (a.wflags) {
+            flag_wait_geq(a.wflags + (int64_t)(ti < 0 ? a.k : ti) * NBLK + NBLK - 1, a.wepoch);
+            if (lane_id() == 0) fence_proxy_async_global();   // panel's generic stores -> bulk copies
+        }
+    };
+    if (ntiles > 0) {
+        wait_tile(tile_of(0));
+        stage_first(sm, vblock(tile_of(0), blk(0)));
+    }
     for (int q = 0; q < ntiles; ++q) {
         const int ti = tile_of(q);
         double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
@@ -326,7 +335,10 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
             const int s = blk(si);
             const double* nxt = nullptr;
             if (si + 1 < NBLK) nxt = vblock(ti, blk(si + 1));
-            else if (q + 1 < ntiles) nxt = vblock(tile_of(q + 1), blk(0));
+            else if (q + 1 < ntiles) {
+                wait_tile(tile_of(q + 1));
+                nxt = vblock(tile_of(q + 1), blk(0));
+            }
             if (ti < 0)
                 apply_block<NB, W, IB, false, TRANS, false, true>(X, sm, vblock(ti, s), Tt + (int64_t)s * IB * IB,
                                                                   nullptr, a.ld, s * IB, nxt, vph);

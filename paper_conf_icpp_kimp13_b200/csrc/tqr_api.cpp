@@ -70,6 +70,7 @@ struct Owner {
     double* sc_Vexp = nullptr;      // nb*nb
     cudaStream_t s_panel = nullptr, s_upd = nullptr, s_comm = nullptr;
     cudaStream_t s_io = nullptr;                    // streamed tqr_factor: per-column H2D + a1, a8 + D2H
+    cudaStream_t s_look = nullptr;                  // lookahead update overlapped with its own panel
     std::vector<cudaEvent_t> ev_load;               // ev_load[lc]: local column lc resident in tile layout
     std::vector<cudaStream_t> s_u;                  // bulk-update streams (column lc -> s_u[lc % S])
     std::vector<cudaEvent_t> ev_panel, ev_recv, ev_look;
@@ -108,6 +109,7 @@ struct tqr_plan_s {
     // streamed tqr_factor (caller A not on the owner's device): column loads overlap the
     // factorization (panel k / the step-0 update of column j wait for ev_load), R of column k is
     // written back on s_io as soon as PANEL(k) completes
+    bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
     bool streamed = false;
     void* sA = nullptr;
     int64_t slda = 0;
@@ -207,6 +209,7 @@ void free_owner(Owner& o) {
     if (o.s_upd) cudaStreamDestroy(o.s_upd);
     if (o.s_comm) cudaStreamDestroy(o.s_comm);
     if (o.s_io) cudaStreamDestroy(o.s_io);
+    if (o.s_look) cudaStreamDestroy(o.s_look);
 }
 
 // Host-side DAG (Fig. 3) per rank, the same order the executor issues.
@@ -285,6 +288,7 @@ tqr_status sync_all(tqr_plan h) {
         CUDA_TRY(h, cudaStreamSynchronize(o.s_comm));
         for (auto su : o.s_u) CUDA_TRY(h, cudaStreamSynchronize(su));
         if (o.s_io) CUDA_TRY(h, cudaStreamSynchronize(o.s_io));
+        if (o.s_look) CUDA_TRY(h, cudaStreamSynchronize(o.s_look));
     }
     return TQR_OK;
 }
@@ -429,6 +433,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->nccl_mode = use_nccl;
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
+    if (const char* e = getenv("TQR_LA_OVERLAP")) h->la_overlap = atoi(e) != 0;
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
     // Tree mode (NEXT-1): TS domains of L tiles factored one per CTA, merged by a flat TT chain.
     // Auto: a single panel column (q == 1, e.g. C4) whose flat chain has parallelism 1.
@@ -493,7 +498,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
             if (h->owner_of[j] == ow.id) { ow.lidx[j] = (int32_t)ow.cols.size(); ow.cols.push_back(j); }
         if (cudaSetDevice(ow.dev) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "cudaSetDevice(%d)", ow.dev));
         auto mk = [&](cudaStream_t* s, int prio) { return cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, prio); };
-        if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi) || mk(&ow.s_io, prio_hi))
+        if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi) || mk(&ow.s_io, prio_hi) ||
+            mk(&ow.s_look, prio_hi))
             return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
         const int S = h->nstreams;
         ow.s_u.assign(S, nullptr);
@@ -642,7 +648,8 @@ struct PanelRefs {
 // (TSMQR against row tile k_head) applied to nslices column slices of X.
 cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const void* Vexp, void* X, int64_t col_stride,
                     int64_t tile_stride, int64_t ld, int group0, int gstride, int k_head, int p_end, int do_unmqr,
-                    int w, int nslices, bool trans, cudaStream_t s, int vstride = 1) {
+                    int w, int nslices, bool trans, cudaStream_t s, int vstride = 1,
+                    const unsigned* wflags = nullptr, unsigned wepoch = 0) {
     if (h->f32()) {
         tqr::UpdateArgsT<float> u;
         u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
@@ -654,6 +661,7 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
     u.V = (const double*)V; u.T = (const double*)T; u.Vexp = (const double*)Vexp; u.X = (double*)X;
     u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
     u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr; u.vstride = vstride;
+    u.wflags = wflags; u.wepoch = wepoch;
     return tqr::launch_update(h->nb, h->ib, w, u, nslices, trans, s);
 }
 // Q_k^T (trans) or Q_k applied to X.  Flat: one launch (UNMQR(k) + TSMQR(k+1..p-1)).  Tree (D > 1
@@ -665,12 +673,12 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
 // reverse order.  Returns the number of launches in *nl.
 cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col_stride, int64_t tile_stride,
                    int64_t ld, int group0, int gstride, int k, int w, int nslices, bool trans, cudaStream_t s,
-                   int64_t* nl = nullptr) {
+                   int64_t* nl = nullptr, const unsigned* wflags = nullptr, unsigned wepoch = 0) {
     const int D = h->ndom(k), L = h->tree_L;
     if (D == 1) {
         if (nl) *nl += 1;
         return update1(h, r.V, r.T, r.Vexp, X, col_stride, tile_stride, ld, group0, gstride, k, h->p, 1, w, nslices,
-                       trans, s);
+                       trans, s, 1, wflags, wepoch);
     }
     auto dom = [&](int d) {
         const int head = k + d * L, end = std::min(head + L, h->p);
@@ -971,13 +979,22 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             const int nloc = (int)D.cols.size();
             const bool la = h->lookahead && first < nloc && D.cols[first] == k + 1;
             if (la) {
-                // lookahead: column k+1 first, on the high-priority panel stream
-                CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, ready, 0));
-                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_u[first % S][k - 1], 0));
-                if (k == 0 && h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_load[first], 0));
+                // lookahead: column k+1 first, on a high-priority stream.  FP64 flat panel of this
+                // owner: the update runs beside PANEL(k) (already enqueued, so its CTAs are
+                // dispatched first) and waits per reflector tile on the panel's flags; otherwise it
+                // follows the whole panel (or the broadcast) on the panel stream.
+                const bool ovl = mine && h->la_overlap && !h->f32() && h->ndom(k) == 1;
+                cudaStream_t sl = ovl ? D.s_look : D.s_panel;
+                if (!ovl) CUDA_TRY(h, cudaStreamWaitEvent(sl, ready, 0));
+                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_u[first % S][k - 1], 0));
+                if (k == 0 && h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_load[first], 0));
                 const int wl = w_look(h);
-                CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, D.s_panel,
-                                   &h->launches));
+                CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, sl,
+                                   &h->launches, ovl ? D.flags : nullptr, epoch0 + (unsigned)k + 1));
+                if (ovl) {   // PANEL(k+1) (panel stream) after the lookahead
+                    CUDA_TRY(h, cudaEventRecord(D.ev_look[k], sl));
+                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_look[k], 0));
+                }
                 first += 1;
             }
             CUDA_TRY(h, cudaEventRecord(D.ev_look[k], D.s_panel));

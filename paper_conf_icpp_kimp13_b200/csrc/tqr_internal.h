@@ -59,6 +59,11 @@ struct UpdateArgsT {
     int k, p;
     int do_unmqr;        // 1: apply Q_kk (UNMQR) to row tile k as well
     int vstride = 1;     // reflector tile i at V + i*vstride*image tile, T + i*vstride*ib*nb
+    // FP64 lookahead overlapped with its panel: before reading reflector tile i (i = k for UNMQR),
+    // wait until the panel kernel has published F(i, last ib block) >= wepoch (every block of tile
+    // i then is, by the panel's release/acquire chain); null = the stream dependency suffices
+    const unsigned* wflags = nullptr;
+    unsigned wepoch = 0;
 };
 using UpdateArgs = UpdateArgsT<double>;
 
