@@ -192,6 +192,8 @@ def main():
     ap.add_argument("--no-lookahead", action="store_true")
     ap.add_argument("--tree", type=int, default=0,
                     help="elimination tree: 0 auto (tree for q == 1), -1 flat TS, L > 0 TS domains of L tiles")
+    ap.add_argument("--solve", type=int, default=0,
+                    help="also time tqr_solve_ls with this many right-hand sides (NEXT-3; 'solve' key)")
     ap.add_argument("--tree-group", type=int, default=0,
                     help="tree merge: 0 auto (two-level for >= 16 domains), -1 flat chain, G > 1 groups of G")
     args = ap.parse_args()
@@ -304,6 +306,35 @@ def main():
                       "R-out + D2H overlapped inside the call"}
         del Ah
 
+    # ---- least squares throughput (NEXT-3): Q^T B (update kernel) + tile back substitution on a
+    # device-resident B of --solve columns; B restored from a pristine copy between calls (untimed)
+    solve = None
+    if args.solve > 0 and world == 1:
+        nr = args.solve
+        gen_b = torch.Generator(device="cuda").manual_seed(seed + 1)
+        B0 = torch.randn((nr, m), dtype=tdt, device="cuda", generator=gen_b).t()
+        Bw = torch.empty((nr, m), dtype=tdt, device="cuda").t()
+        plan.load(A0)
+        plan.factor_tiles()
+        Bw.copy_(B0)
+        plan.solve_ls(Bw)
+        torch.cuda.synchronize()
+        st = 0.0
+        for _ in range(K):
+            Bw.copy_(B0)
+            torch.cuda.synchronize()
+            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s0.record(stream)
+            plan.solve_ls(Bw)
+            s1.record(stream)
+            torch.cuda.synchronize()
+            st += s0.elapsed_time(s1)
+        sms = st / K
+        sfl = (4.0 * m * n - 1.0 * n * n) * nr      # Q^T B (4mn - 2n^2) + back substitution (n^2) per RHS
+        solve = {"nrhs": nr, "ms": round(sms, 3), "gflops": round(sfl / (sms * 1e-3) / 1e9, 3),
+                 "flops": "(4mn - n^2) nrhs: Householder Q^T B (4mn - 2n^2) + tile back substitution (n^2)"}
+        del B0, Bw
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle
@@ -357,6 +388,8 @@ def main():
             "e2e": e2e,
             "cpu_baseline": cpu,
         }
+        if solve is not None:
+            line["solve"] = solve
         print(json.dumps(line), flush=True)
     plan.close()
     if dist is not None:

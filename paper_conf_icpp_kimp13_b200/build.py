@@ -25,6 +25,7 @@ COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-I" + os.pat
 SOURCES = [
     os.path.join(CSRC, "kernels", "qr_kernels.cu"),
     os.path.join(CSRC, "kernels", "qr_kernels_f32.cu"),
+    os.path.join(CSRC, "kernels", "trsm.cu"),
     os.path.join(CSRC, "tqr_api.cpp"),
 ]
 

@@ -12,7 +12,7 @@
 //                   "top" row block of every TS pair.  Also used (TRANS / reverse order) for
 //                   Q^T B and Q B in tqr_apply_qt.
 //   layout kernels: column-major <-> tile-major (128-bit when aligned), R out with zeroed
-//                   lower part, and the back substitution of tqr_solve_ls (Eq. 3).
+//                   lower part (the back substitution of tqr_solve_ls is in trsm.cu).
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
@@ -295,10 +295,19 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     auto& sm = *reinterpret_cast<Smem<NB, W, IB, false>*>(smem_raw);
     constexpr int SPG = NB / W;     // slices per column group
     constexpr int NBLK = NB / IB;
-    const int grp = blockIdx.x / SPG;
-    const int c0 = (blockIdx.x % SPG) * W;
+    // wavefront apply (nsteps > 1): CTA = (step offset st, slice); step k = a.k +- st with its own
+    // reflector column (V, T, Vexp + k * column strides); tile i of step k waits until the
+    // previous step's CTA of the same slice has finished tile i (progress flags, lower CTA index)
+    const int st = a.nsteps > 1 ? (int)(blockIdx.x / a.nslc) : 0;
+    const int bid = a.nsteps > 1 ? (int)(blockIdx.x % a.nslc) : (int)blockIdx.x;
+    const int k = TRANS ? a.k + st : a.k - st;
+    const double* __restrict__ Vb = a.V + (int64_t)st * (TRANS ? 1 : -1) * a.vcol;
+    const double* __restrict__ Tb = a.T + (int64_t)st * (TRANS ? 1 : -1) * a.tcol;
+    const double* __restrict__ Eb = a.Vexp + (int64_t)st * (TRANS ? 1 : -1) * a.ecol;
+    const int grp = bid / SPG;
+    const int c0 = (bid % SPG) * W;
     double* Xg = a.X + (int64_t)(a.group0 + grp * a.gstride) * a.col_stride + (int64_t)c0 * a.ld;
-    double* Xk = Xg + (int64_t)a.k * a.tile_stride;
+    double* Xk = Xg + (int64_t)k * a.tile_stride;
     const int64_t vtile = (int64_t)NB * NB;
     Slice<NB, W, IB> X;
     stage_init(sm);
@@ -307,18 +316,27 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     // Reflector blocks in application order; block q of the sequence is staged (cp.async) while
     // block q-1's GEMM2 runs.  Forward: UNMQR blocks 0..NBLK-1, then for i = k+1..p-1 blocks
     // 0..NBLK-1 of V_i.  Backward: i = p-1..k+1 blocks NBLK-1..0, then UNMQR blocks NBLK-1..0.
-    const int ntiles = a.p - a.k - 1 + (a.do_unmqr ? 1 : 0);
+    const int ntiles = a.p - k - 1 + (a.do_unmqr ? 1 : 0);
     auto tile_of = [&](int q) -> int {            // q-th tile of the sequence; -1 = UNMQR (row tile k)
-        if (TRANS) return a.do_unmqr ? (q == 0 ? -1 : a.k + q) : a.k + 1 + q;
-        return (q < a.p - a.k - 1) ? a.p - 1 - q : -1;
+        if (TRANS) return a.do_unmqr ? (q == 0 ? -1 : k + q) : k + 1 + q;
+        return (q < a.p - k - 1) ? a.p - 1 - q : -1;
     };
     auto vblock = [&](int ti, int s) -> const double* {
-        return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;
+        return (ti < 0 ? Eb : Vb + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;
+    };
+    // progress of the previous step's CTA needed before row tile ti: forward, the previous step
+    // (k-1) runs k-1, k, k+1, ..; backward (Q), the previous step (k+1) runs p-1, .., k+1
+    auto wait_prev = [&](int ti) {
+        if (st > 0 && !(!TRANS && ti < 0)) {      // backward UNMQR row k: untouched by step k+1
+            const int row = ti < 0 ? k : ti;
+            const unsigned need = TRANS ? (unsigned)(row - k + 2) : (unsigned)(a.p - row);
+            flag_wait_geq(a.prog + (int64_t)(st - 1) * a.nslc + bid, need);
+        }
     };
     auto blk = [&](int si) { return TRANS ? si : NBLK - 1 - si; };
     auto wait_tile = [&](int ti) {   // lookahead overlapped with the panel: tile ti published?
         if (a.wflags) {
-            flag_wait_geq(a.wflags + (int64_t)(ti < 0 ? a.k : ti) * NBLK + NBLK - 1, a.wepoch);
+            flag_wait_geq(a.wflags + (int64_t)(ti < 0 ? k : ti) * NBLK + NBLK - 1, a.wepoch);
             if (lane_id() == 0) fence_proxy_async_global();   // panel's generic stores -> bulk copies
         }
     };
@@ -329,8 +347,13 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     for (int q = 0; q < ntiles; ++q) {
         const int ti = tile_of(q);
         double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
-        const double* Tt = a.T + (int64_t)(ti < 0 ? a.k : ti * a.vstride) * IB * NB;
-        X.load(Xi, a.ld);
+        const double* Tt = Tb + (int64_t)(ti < 0 ? k : ti * a.vstride) * IB * NB;
+        if (a.nsteps > 1) {
+            wait_prev(ti);
+            X.load_cg(Xi, a.ld);     // written by another CTA: L2, not a stale L1 line
+        } else {
+            X.load(Xi, a.ld);
+        }
         for (int si = 0; si < NBLK; ++si) {
             const int s = blk(si);
             const double* nxt = nullptr;
@@ -347,7 +370,9 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
                                                                    Xk + s * IB, a.ld, 0, nxt, vph);
         }
         X.store(Xi, a.ld);
+        if (a.nsteps > 1) __threadfence();
         __syncthreads();   // row tile k (the TS "top") is re-read by other threads
+        if (a.nsteps > 1 && threadIdx.x == 0) flag_release(a.prog + (int64_t)st * a.nslc + bid, (unsigned)(q + 1));
     }
 }
 
@@ -416,29 +441,6 @@ __global__ void from_tiles_kernel(T* __restrict__ dst, int64_t lda, int64_t dst_
             __stcs(reinterpret_cast<float4*>(d + r), make_float4(v[0], v[1], v[2], v[3]));
         }
     }
-}
-
-// Back substitution R X = C for the n x n upper-triangular R (gathered column-major into R,
-// ld = ldr).  One CTA per right-hand side; columns of R are streamed (Eq. 3).
-template <class T>
-__global__ void trsv_upper_kernel(const T* __restrict__ R, int64_t ldr, T* __restrict__ C, int64_t ldc, int64_t n) {
-    T* x = C + (int64_t)blockIdx.x * ldc;
-    __shared__ T xi_s;
-    for (int64_t i = n - 1; i >= 0; --i) {
-        if (threadIdx.x == 0) xi_s = x[i] / R[i + i * ldr];
-        __syncthreads();
-        const T xi = xi_s;
-        const T* rc = R + i * ldr;
-        for (int64_t r = threadIdx.x; r < i; r += blockDim.x) x[r] -= rc[r] * xi;
-        if (threadIdx.x == 0) x[i] = xi;
-        __syncthreads();
-    }
-}
-
-template <class T>
-__global__ void zero_diag_check_kernel(const T* __restrict__ R, int64_t ldr, int64_t n, int64_t* first_zero) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        if (R[i + i * ldr] == T(0)) atomicMin(reinterpret_cast<unsigned long long*>(first_zero), (unsigned long long)i);
 }
 
 // ============================================================================ launchers
@@ -592,23 +594,6 @@ template cudaError_t launch_from_tiles<double>(double*, int64_t, int64_t, const 
                                                int64_t, int, int64_t, int64_t, int, cudaStream_t);
 template cudaError_t launch_from_tiles<float>(float*, int64_t, int64_t, const float*, const int32_t*, int,
                                               int64_t, int, int64_t, int64_t, int, cudaStream_t);
-
-template <class T>
-cudaError_t launch_trsv_upper(const T* R, int64_t ldr, T* C, int64_t ldc, int64_t n, int64_t nrhs, cudaStream_t s) {
-    if (nrhs <= 0) return cudaSuccess;
-    trsv_upper_kernel<T><<<(unsigned)nrhs, 256, 0, s>>>(R, ldr, C, ldc, n);
-    return cudaGetLastError();
-}
-
-template <class T>
-cudaError_t launch_zero_diag_check(const T* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s) {
-    zero_diag_check_kernel<T><<<64, 256, 0, s>>>(R, ldr, n, first_zero);
-    return cudaGetLastError();
-}
-template cudaError_t launch_trsv_upper<double>(const double*, int64_t, double*, int64_t, int64_t, int64_t, cudaStream_t);
-template cudaError_t launch_trsv_upper<float>(const float*, int64_t, float*, int64_t, int64_t, int64_t, cudaStream_t);
-template cudaError_t launch_zero_diag_check<double>(const double*, int64_t, int64_t, int64_t*, cudaStream_t);
-template cudaError_t launch_zero_diag_check<float>(const float*, int64_t, int64_t, int64_t*, cudaStream_t);
 
 size_t panel_smem_bytes(int nb, int ib) {
 #define TQR_PS(NB_, IB_) if (nb == NB_ && ib == IB_) return sizeof(Smem<NB_, IB_, IB_, true>);

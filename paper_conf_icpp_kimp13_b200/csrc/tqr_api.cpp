@@ -109,6 +109,8 @@ struct tqr_plan_s {
     // streamed tqr_factor (caller A not on the owner's device): column loads overlap the
     // factorization (panel k / the step-0 update of column j wait for ev_load), R of column k is
     // written back on s_io as soon as PANEL(k) completes
+    void* prog = nullptr;           // wavefront apply progress flags (q * nslices)
+    size_t prog_n = 0;
     bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
     bool streamed = false;
     void* sA = nullptr;
@@ -128,7 +130,6 @@ struct tqr_plan_s {
     // apply / solve workspace (single-device plans)
     void* bw = nullptr;
     size_t bw_elems = 0;
-    void* rcm = nullptr;
     int64_t* dflag = nullptr;
 
     bool nccl_mode = false;         // one process per GPU, panels broadcast with NCCL
@@ -387,8 +388,8 @@ tqr_status tqr_destroy(tqr_plan h) {
     if (h->comm && h->nccl) h->nccl->CommDestroy(h->comm);
     if (!h->owners.empty()) cudaSetDevice(h->owners[0].dev);
     if (h->bw) cudaFree(h->bw);
-    if (h->rcm) cudaFree(h->rcm);
     if (h->dflag) cudaFree(h->dflag);
+    if (h->prog) cudaFree(h->prog);
     for (auto& o : h->owners) free_owner(o);
     cudaGetLastError();
     delete h;
@@ -1150,9 +1151,35 @@ static tqr_status single_device(tqr_plan h, int* dev) {
 }
 
 // Bw (mp x 32*nslices, ld ldw) <- Q^T Bw (forward over the panels) or Q Bw (reverse).
+// FP64, one owner, flat tree: all q steps in one wavefront launch (step k+1's chain follows step
+// k's tile by tile), otherwise one launch per step.
 static tqr_status apply_device(tqr_plan h, char trans, void* Bw, int64_t ldw, int64_t nslices, cudaStream_t s) {
     const int q = h->q, nb = h->nb;
     const bool fwd = (trans == 'T' || trans == 't');
+    if (!h->f32() && h->tree_L == 0 && h->owners.size() == 1 && q > 1 && !getenv("TQR_NO_WAVEFRONT_APPLY")) {
+        Owner& O = h->owners[0];
+        const size_t need = (size_t)q * nslices;
+        if (need > h->prog_n) {
+            if (h->prog) cudaFree(h->prog);
+            h->prog = nullptr;
+            h->prog_n = 0;
+            CUDA_TRY(h, cudaMalloc(&h->prog, need * sizeof(unsigned)));
+            h->prog_n = need;
+        }
+        CUDA_TRY(h, cudaMemsetAsync(h->prog, 0, need * sizeof(unsigned), s));
+        const int k0 = fwd ? 0 : q - 1;
+        const PanelRefs r = own_refs(h, O, O.lidx[k0]);
+        const int64_t p = h->p;
+        tqr::UpdateArgs u;
+        u.V = (const double*)r.V; u.T = (const double*)r.T; u.Vexp = (const double*)r.Vexp; u.X = (double*)Bw;
+        u.col_stride = (int64_t)nb * ldw; u.tile_stride = nb; u.ld = ldw;
+        u.group0 = 0; u.gstride = 1; u.k = k0; u.p = h->p; u.do_unmqr = 1;
+        u.nsteps = q; u.nslc = (int)nslices; u.prog = (unsigned*)h->prog;
+        u.vcol = p * h->vt; u.tcol = p * (int64_t)h->ib * nb; u.ecol = h->vt;
+        CUDA_TRY(h, tqr::launch_update(nb, h->ib, 32, u, (int)(q * nslices), fwd, s));
+        h->launches++;
+        return TQR_OK;
+    }
     for (int s_ = 0; s_ < q; ++s_) {
         const int k = fwd ? s_ : q - 1 - s_;
         Owner* O = h->local(h->owner_of[k]);
@@ -1227,26 +1254,33 @@ tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
     const int64_t mp = (int64_t)h->p * h->nb;
     st = apply_device(h, 'T', h->bw, mp, nsl, s);
     if (st) return st;
-    // gather R (n x n, column-major) from every owner
+    // R X = (Q^T B)(0:n, :) by tile back substitution on the tile storage (trsm.cu): exact zero on
+    // the diagonal first (LAPACK dtrtrs convention: TQR_ERR_SINGULAR, B unspecified)
     const int64_t n = h->n, nb = h->nb;
-    if (!h->rcm) CUDA_TRY(h, cudaMalloc(&h->rcm, es * (size_t)n * n));
+    const int64_t colsz = (int64_t)h->p * nb * nb;
     if (!h->dflag) CUDA_TRY(h, cudaMalloc(&h->dflag, sizeof(int64_t)));
+    const unsigned long long big = ~0ull;
+    CUDA_TRY(h, cudaMemcpyAsync(h->dflag, &big, sizeof(big), cudaMemcpyHostToDevice, s));
     for (auto& o : h->owners) {
-        if (o.cols.empty()) continue;
-        CUDA_TRY(h, from_tiles(h, h->rcm, n, nb * n, o.tiles, o.cols_dev, (int)o.cols.size(), n, n, 0, s));
+        const int nc = (int)o.cols.size();
+        auto* fz = reinterpret_cast<unsigned long long*>(h->dflag);
+        if (h->f32()) CUDA_TRY(h, tqr::launch_diag_zero_tiles<float>((const float*)o.tiles, o.cols_dev, nc, colsz, (int)nb, n, fz, s));
+        else CUDA_TRY(h, tqr::launch_diag_zero_tiles<double>((const double*)o.tiles, o.cols_dev, nc, colsz, (int)nb, n, fz, s));
         h->launches++;
     }
-    const int64_t big = INT64_MAX;
-    CUDA_TRY(h, cudaMemcpyAsync(h->dflag, &big, sizeof(int64_t), cudaMemcpyHostToDevice, s));
-    if (h->f32()) CUDA_TRY(h, tqr::launch_zero_diag_check<float>((const float*)h->rcm, n, n, h->dflag, s));
-    else CUDA_TRY(h, tqr::launch_zero_diag_check<double>((const double*)h->rcm, n, n, h->dflag, s));
-    int64_t first_zero = 0;
-    CUDA_TRY(h, cudaMemcpyAsync(&first_zero, h->dflag, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    unsigned long long first_zero = 0;
+    CUDA_TRY(h, cudaMemcpyAsync(&first_zero, h->dflag, sizeof(first_zero), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
-    if (first_zero != big) return fail(h, TQR_ERR_SINGULAR, "R(%lld,%lld) == 0", (long long)first_zero, (long long)first_zero);
-    if (h->f32()) CUDA_TRY(h, tqr::launch_trsv_upper<float>((const float*)h->rcm, n, (float*)h->bw, mp, n, nrhs, s));
-    else CUDA_TRY(h, tqr::launch_trsv_upper<double>((const double*)h->rcm, n, (double*)h->bw, mp, n, nrhs, s));
-    h->launches++;
+    if (first_zero != big) return fail(h, TQR_ERR_SINGULAR, "R(%llu,%llu) == 0", first_zero, first_zero);
+    for (int i = h->q - 1; i >= 0; --i) {
+        Owner* O = h->local(h->owner_of[i]);
+        const void* Rcol = h->at(O->tiles, (int64_t)O->lidx[i] * colsz);
+        if (h->f32())
+            CUDA_TRY(h, tqr::launch_trsm_step<float>((int)nb, (const float*)Rcol, i, (float*)h->bw, mp, n, (int)nsl, s));
+        else
+            CUDA_TRY(h, tqr::launch_trsm_step<double>((int)nb, (const double*)Rcol, i, (double*)h->bw, mp, n, (int)nsl, s));
+        h->launches += (i > 0) ? 2 : 1;
+    }
     CUDA_TRY(h, cudaMemcpy2DAsync(B, ldb * es, h->bw, mp * es, n * es, nrhs, cudaMemcpyDefault, s));
     CUDA_TRY(h, cudaStreamSynchronize(s));
     return TQR_OK;

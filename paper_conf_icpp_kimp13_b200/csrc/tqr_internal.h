@@ -64,6 +64,14 @@ struct UpdateArgsT {
     // i then is, by the panel's release/acquire chain); null = the stream dependency suffices
     const unsigned* wflags = nullptr;
     unsigned wepoch = 0;
+    // FP64 wavefront apply of nsteps consecutive panels in one launch (tqr_apply_qt / solve_ls,
+    // single owner, flat tree): grid = nsteps * nslc CTAs, step offset st = CTA / nslc processes
+    // step k +- st (TRANS: +) with V, T, Vexp advanced by st * (vcol, tcol, ecol) elements; prog
+    // (nsteps * nslc, zeroed) counts the chain tiles each CTA has finished
+    int nsteps = 1;
+    int nslc = 0;
+    int64_t vcol = 0, tcol = 0, ecol = 0;
+    unsigned* prog = nullptr;
 };
 using UpdateArgs = UpdateArgsT<double>;
 
@@ -84,10 +92,14 @@ template <class T>
 cudaError_t launch_from_tiles(T* dst, int64_t lda, int64_t dst_group_stride, const T* src, const int32_t* cols_dev,
                               int ncols, int64_t src_col_stride, int nb, int64_t m_rows, int64_t n_valid,
                               int local_dst, cudaStream_t s);
+// Step i of the tile back substitution (trsm.cu): X_i = R_ii^-1 C_i, then C_r -= R_ri X_i, r < i.
+// Rcol = column tile i of R in tile storage (tile r at Rcol + r*nb*nb); C = mp x 32*nslices, ld ldc.
 template <class T>
-cudaError_t launch_trsv_upper(const T* R, int64_t ldr, T* C, int64_t ldc, int64_t n, int64_t nrhs, cudaStream_t s);
+cudaError_t launch_trsm_step(int nb, const T* Rcol, int i, T* C, int64_t ldc, int64_t n, int nslices, cudaStream_t s);
+// atomicMin of the first global diagonal index g < n with R(g, g) == 0 over the owned column tiles
 template <class T>
-cudaError_t launch_zero_diag_check(const T* R, int64_t ldr, int64_t n, int64_t* first_zero, cudaStream_t s);
+cudaError_t launch_diag_zero_tiles(const T* tiles, const int32_t* cols_dev, int ncols, int64_t colsz, int nb, int64_t n,
+                                   unsigned long long* first_zero, cudaStream_t s);
 
 // ---- FP32 path (kernels/qr_kernels_f32.cu)
 // FFMA trailing update; V / Vexp are FP32 stage images (f32_img_tile elements per tile)

@@ -165,6 +165,49 @@ def test_solve_ls_matches_oracle():
     np.testing.assert_allclose(X, Xo, rtol=1e-9, atol=1e-11)
 
 
+@pytest.mark.parametrize("m,n,nb,ib,nrhs", [
+    (1024, 1024, 512, 32, 1),       # 2 tile rows, one RHS
+    (1536, 1024, 256, 32, 70),      # tall, 3 RHS slices (ragged last slice)
+    (700, 650, 128, 32, 33),        # ragged rows, columns and RHS (padded diagonal rows)
+    (640, 640, 64, 16, 100),        # nb = 64: update row blocks straddle tiles
+])
+def test_tile_trsm_solve_matches_oracle(m, n, nb, ib, nrhs):
+    """tqr_solve_ls = Q^T B on the update kernel + the tile back substitution (trsm.cu: inverted
+    32 x 32 diagonal blocks inside each R_ii, FMA updates of the rows above) vs the oracle's
+    Eqs. (2)-(3) (plain back substitution)."""
+    A = synthetic.gaussian(m, n, 7000 + m + n)
+    B = synthetic.gaussian(m, nrhs, 7100 + nrhs)
+    plan, _ = gpu_qr(A, nb, ib)
+    Bd = dev_colmajor(B)
+    plan.solve_ls(Bd)
+    X = to_np(Bd)[:n]
+    Xo = oracle.solve_ls(A, B)
+    np.testing.assert_allclose(X, Xo, rtol=1e-8, atol=1e-10 * max(1.0, np.abs(Xo).max()))
+    plan.close()
+
+
+@pytest.mark.parametrize("m,n,nb,ib,nrhs", [(1536, 1024, 256, 32, 40), (640, 600, 64, 16, 7), (2048, 2048, 512, 32, 96)])
+def test_wavefront_apply_bitwise(m, n, nb, ib, nrhs, monkeypatch):
+    """One-launch wavefront Q^T B / Q B (step k+1's CTA follows step k's tile by tile on progress
+    flags) computes every chain exactly as the per-step launches: bitwise equal, and Q (Q^T B) = B."""
+    A = synthetic.gaussian(m, n, 7300 + m)
+    B = synthetic.gaussian(m, nrhs, 7400 + nrhs)
+    plan, _ = gpu_qr(A, nb, ib)
+    out = {}
+    for mode in ("wave", "steps"):
+        if mode == "steps":
+            monkeypatch.setenv("TQR_NO_WAVEFRONT_APPLY", "1")
+        Bd = dev_colmajor(B)
+        plan.apply_qt(Bd, "T")
+        QtB = to_np(Bd)
+        plan.apply_qt(Bd, "N")
+        out[mode] = (QtB, to_np(Bd))
+    assert np.array_equal(out["wave"][0], out["steps"][0])
+    assert np.array_equal(out["wave"][1], out["steps"][1])
+    np.testing.assert_allclose(out["wave"][1], B, atol=1e-12)
+    plan.close()
+
+
 def test_host_pointer_and_pinned_paths_match_device():
     m, n, nb, ib = 384, 256, 64, 16
     A = synthetic.gaussian(m, n, 81)
