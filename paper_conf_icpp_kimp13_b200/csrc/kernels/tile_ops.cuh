@@ -414,9 +414,10 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
 #pragma unroll
                 for (int nf = 0; nf < G::NF; ++nf) ss += xv[nf][0] * xv[nf][0] + xv[nf][1] * xv[nf][1];
             }
+            // column groups mf < mfc hold columns j < c only (finished): no dots, no update
             double pd[G::MF], p0[G::MF];
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) {
+            for (int mf = mfc; mf < G::MF; ++mf) {
                 double sdot = 0.0, sdiag = 0.0;
 #pragma unroll
                 for (int nf = 0; nf < G::NF; ++nf)
@@ -439,7 +440,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             if (t == 0) {
                 double* rec = fbp + wq * FBW;
 #pragma unroll
-                for (int mf = 0; mf < G::MF; ++mf) {
+                for (int mf = mfc; mf < G::MF; ++mf) {
                     rec[mf * 8 + g] = pd[mf];
                     if (GE) rec[IB + mf * 8 + g] = p0[mf];
                 }
@@ -464,7 +465,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = scale x (+ e_d)
             double tw[G::MF];
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) {
+            for (int mf = mfc; mf < G::MF; ++mf) {
                 const int j = mf * 8 + g;
                 tw[mf] = 0.0;
                 if (j > c) {
@@ -481,7 +482,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 }
             }
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) {
+            for (int mf = mfc; mf < G::MF; ++mf) {
 #pragma unroll
                 for (int nf = 0; nf < G::NF; ++nf)
 #pragma unroll
