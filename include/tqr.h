@@ -112,7 +112,10 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
  * its upper triangle and every entry below the diagonal of A is zero (the reflectors stay
  * inside the plan in tile layout for tqr_apply_qt / tqr_solve_ls).  In multi-process mode
  * A is the full matrix on every rank and each rank writes back the columns it owns.
- * The call runs a1 (layout convert), a2-a7 (tiled factorisation) and a8 (R out).
+ * The call runs a1 (layout convert), a2-a7 (tiled factorisation) and a8 (R out).  When A is
+ * not resident on the owning device (host memory or another GPU), the column loads and the R
+ * stores are pipelined with the factorisation (column k is written back as soon as its panel
+ * is factored); the result is bitwise the same.
  */
 tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda);
 
@@ -131,8 +134,9 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda);
 tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs);
 
 /*
- * Least squares min ||A X - B||_F via Eqs. (2)-(3): B <- Q^T B, then R X = B(0:n, :) by
- * back substitution; X is returned in B(0:n, :) (rows n..m-1 unspecified).
+ * Least squares min ||A X - B||_F via Eqs. (2)-(3): B <- Q^T B, then R X = B(0:n, :) by tile
+ * back substitution on the resident R tiles; X is returned in B(0:n, :) (rows
+ * n..m-1 unspecified).  B may be host or device memory (ldb >= m).
  * TQR_ERR_SINGULAR if some R_ii == 0 exactly (B unspecified).
  */
 tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs);
