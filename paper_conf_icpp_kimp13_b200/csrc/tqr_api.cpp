@@ -100,7 +100,9 @@ struct tqr_plan_s {
     bool logical = false;
     int rank = 0, world = 1;
     bool lookahead = true, profile = false;
-    int nstreams = 4;               // bulk-update streams per owner (TQR_UPDATE_STREAMS)
+    int nstreams = 4;               // bulk-update streams per owner (TQR_UPDATE_STREAMS), column lc -> lc % S
+    int nstreams_io = 8;            // streamed factor: contiguous column chunks, one stream each
+    int nstreams_alloc() const { return std::max(nstreams, nstreams_io); }
     int panel_split = 1;            // sub-slice CTAs per ib column block in the panel kernel
     int tree_L = 0;                 // TS-domain length (tiles); 0 = flat TS chain
     int dmax = 1;                   // max domains of any step = ceil(p / tree_L)
@@ -502,7 +504,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi) || mk(&ow.s_io, prio_hi) ||
             mk(&ow.s_look, prio_hi))
             return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
-        const int S = h->nstreams;
+        const int S = h->nstreams_alloc();
         ow.s_u.assign(S, nullptr);
         for (auto& su : ow.s_u)
             if (mk(&su, prio_lo)) return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
@@ -866,7 +868,12 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
 tqr_status tqr_factor_tiles(tqr_plan h) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
-    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib, S = h->nstreams;
+    const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
+    // bulk-update streams: round-robin (column lc on stream lc % S) for resident data; a streamed
+    // factor maps contiguous chunks of columns to streams instead, so the early chunks run through
+    // their steps while later columns are still being copied in (round-robin would block every
+    // stream's step-1 launch behind its last column's load)
+    const int S = h->streamed ? h->nstreams_io : h->nstreams;
     const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile, vt = h->vt;
     const unsigned epoch0 = h->epoch;
     h->epoch += (unsigned)q + 1;
@@ -880,6 +887,9 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             CUDA_TRY(h, cudaEventRecord(o.tref[0], o.s_panel));
         }
     }
+    auto stream_of = [&](int lc, int nloc) -> int {
+        return h->streamed ? (int)(((int64_t)lc * S) / nloc) : lc % S;
+    };
     auto wait_all_u = [&](Owner& D, cudaStream_t st, int kk) -> tqr_status {
         for (int u = 0; u < S; ++u) CUDA_TRY(h, cudaStreamWaitEvent(st, D.ev_u[u][kk], 0));
         return TQR_OK;
@@ -987,7 +997,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 const bool ovl = mine && h->la_overlap && !h->f32() && h->ndom(k) == 1;
                 cudaStream_t sl = ovl ? D.s_look : D.s_panel;
                 if (!ovl) CUDA_TRY(h, cudaStreamWaitEvent(sl, ready, 0));
-                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_u[first % S][k - 1], 0));
+                if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_u[stream_of(first, (int)D.cols.size())][k - 1], 0));
                 if (k == 0 && h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_load[first], 0));
                 const int wl = w_look(h);
                 CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, sl,
@@ -1002,8 +1012,17 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             // bulk: columns lc in [first, nloc) with lc % S == u on stream u (stream order chains
             // column lc's step k-1 -> k updates; steps overlap across streams)
             for (int uu = 0; uu < S; ++uu) {
-                int g0 = first + ((uu - first % S) + S) % S;
-                const int ng = (g0 < nloc) ? (nloc - g0 + S - 1) / S : 0;
+                int g0, ng, gs;
+                if (h->streamed) {   // chunk [lo, hi) of the local columns
+                    const int lo = (int)(((int64_t)uu * nloc + S - 1) / S), hi = (int)(((int64_t)(uu + 1) * nloc + S - 1) / S);
+                    g0 = std::max(lo, first);
+                    ng = std::max(0, hi - g0);
+                    gs = 1;
+                } else {
+                    g0 = first + ((uu - first % S) + S) % S;
+                    ng = (g0 < nloc) ? (nloc - g0 + S - 1) / S : 0;
+                    gs = S;
+                }
                 cudaStream_t su = D.s_u[uu];
                 if (ng > 0) {
                     CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
@@ -1011,13 +1030,13 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     const int wb = w_bulk(h);
                     if (k == 0 && h->streamed) {
                         // step 0 of a streamed factor: one launch per column, each after its load
-                        for (int c = g0; c < nloc; c += S) {
+                        for (int c = g0; c < g0 + ng * gs; c += gs) {
                             CUDA_TRY(h, cudaStreamWaitEvent(su, D.ev_load[c], 0));
-                            CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, c, S, k, wb, nb / wb, true, su,
+                            CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, c, gs, k, wb, nb / wb, true, su,
                                                &h->launches));
                         }
                     } else {
-                        CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, S, k, wb, ng * (nb / wb), true, su,
+                        CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, gs, k, wb, ng * (nb / wb), true, su,
                                            &h->launches));
                     }
                     if (h->profile) {
