@@ -172,6 +172,31 @@ tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const in
  * (capacity cap) and the length to *len. */
 tqr_status tqr_generate_guide(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len);
 
+/* Measured average time (seconds) of one tile operation on a device (the paper's time_i(op),
+ * P:L878-881): T = triangulation (GEQRT), E = elimination (TSQRT), UT = update for
+ * triangulation (UNMQR), UE = update for elimination (TSMQR). */
+typedef struct {
+    double t_T, t_E, t_UT, t_UE;
+} tqr_tile_times;
+
+/* Main computing device selection, Algorithm 2 (reading Q22): the candidates can
+ * finish T before every other device's UE and E before every other device's UT; the candidate
+ * with the minimum update speed 1/(t_UT + t_UE) is returned (lowest ID on ties); no candidate
+ * -> the fastest updater.  Host-only.  TQR_ERR_ARG on ndev < 1 / negative times. */
+tqr_status tqr_select_main(int32_t ndev, const tqr_tile_times* t, int32_t* main_dev);
+
+/* Number-of-devices selection, Algorithm 3 with Eqs. (10)-(11) (readings
+ * Q23-Q25).  M x N tile grid of T x T tiles, elem_size bytes per element; t[ndev] per-tile
+ * times; speed = ndev x ndev row-major link speeds in bytes/s (speed[x*ndev + y]: x -> y, > 0
+ * off the diagonal; the diagonal is ignored = infinite); main_dev from tqr_select_main.
+ * Outputs: order[ndev] (optional) = the device list (main first, then descending update
+ * speed); Tp[ndev] (optional) = the predicted first-iteration time T(p) = Top(p) + Tcomm(p) for
+ * p = 1..ndev (seconds); *pbest = the p minimising T(p): the first p devices of `order`
+ * participate, distributed by tqr_generate_guide over their rates.  Host-only. */
+tqr_status tqr_select_ndev(int32_t M, int32_t N, int32_t T, int32_t elem_size, int32_t ndev,
+                           const tqr_tile_times* t, const double* speed, int32_t main_dev, int32_t* order,
+                           double* Tp, int32_t* pbest);
+
 /* Device-time statistics of the plan's kernels since the last reset (opt.profile = 1):
  * which = 0 update (UNMQR+TSMQR) kernel, 1 panel (GEQRT+TSQRT) kernel, 2 layout kernels,
  * 3 broadcast.  *count launches, *ms summed CUDA-event milliseconds, *flops algorithmic

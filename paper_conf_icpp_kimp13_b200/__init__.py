@@ -37,6 +37,11 @@ class Options(ctypes.Structure):
                 ("tree_domain", ctypes.c_int32), ("tree_group", ctypes.c_int32)]
 
 
+class TileTimes(ctypes.Structure):
+    _fields_ = [("t_T", ctypes.c_double), ("t_E", ctypes.c_double), ("t_UT", ctypes.c_double),
+                ("t_UE", ctypes.c_double)]
+
+
 _lib = None
 
 
@@ -66,12 +71,15 @@ def lib():
         L.tqr_owner.restype = i32
         L.tqr_schedule.argtypes = [i64, i64, i32, i32, P(i32), i32, i32, P(i32), i64, P(i64)]
         L.tqr_generate_guide.argtypes = [P(i32), i32, P(i32), i32, P(i32)]
+        L.tqr_select_main.argtypes = [i32, P(TileTimes), P(i32)]
+        L.tqr_select_ndev.argtypes = [i32, i32, i32, i32, i32, P(TileTimes), P(ctypes.c_double), i32, P(i32),
+                                      P(ctypes.c_double), P(i32)]
         L.tqr_kernel_stats.argtypes = [vp, i32, P(i64), P(ctypes.c_double), P(ctypes.c_double), i32]
         L.tqr_launch_count.argtypes = [vp]
         L.tqr_launch_count.restype = i64
         for f in ("tqr_create", "tqr_create_ex", "tqr_factor", "tqr_load", "tqr_factor_tiles", "tqr_store_r",
                   "tqr_apply_qt", "tqr_solve_ls", "tqr_destroy", "tqr_nccl_unique_id", "tqr_schedule",
-                  "tqr_generate_guide", "tqr_kernel_stats"):
+                  "tqr_generate_guide", "tqr_kernel_stats", "tqr_select_main", "tqr_select_ndev"):
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -80,7 +88,7 @@ def lib():
 EXPORTED = ["tqr_create", "tqr_create_ex", "tqr_factor", "tqr_load", "tqr_factor_tiles", "tqr_store_r",
             "tqr_apply_qt", "tqr_solve_ls", "tqr_destroy", "tqr_status_string", "tqr_last_error",
             "tqr_nccl_unique_id", "tqr_owner", "tqr_schedule", "tqr_generate_guide", "tqr_kernel_stats",
-            "tqr_launch_count"]
+            "tqr_launch_count", "tqr_select_main", "tqr_select_ndev"]
 
 
 def _check(st: int, h=None):
@@ -201,6 +209,32 @@ def tqr_schedule(m, n, nb, ndev, guide, rank):
     buf = (ctypes.c_int32 * (5 * cnt.value))()
     _check(lib().tqr_schedule(m, n, nb, ndev, g, glen, rank, buf, cnt.value, ctypes.byref(cnt)), None)
     return [tuple(buf[5 * i: 5 * i + 5]) for i in range(cnt.value)]
+
+
+def _times(times):
+    arr = (TileTimes * len(times))()
+    for i, t in enumerate(times):
+        arr[i] = TileTimes(*[float(x) for x in t])
+    return arr
+
+
+def tqr_select_main(times):
+    """Algorithm 2: times = [(t_T, t_E, t_UT, t_UE), ...] per device -> main device id."""
+    out = ctypes.c_int32()
+    _check(lib().tqr_select_main(len(times), _times(times), ctypes.byref(out)), None)
+    return out.value
+
+
+def tqr_select_ndev(M, N, T, elem_size, times, speed, main_dev):
+    """Algorithm 3 + Eqs. (10)-(11): -> (order, [T(p) for p = 1..ndev], p_best)."""
+    nd = len(times)
+    sp = (ctypes.c_double * (nd * nd))(*[float(speed[x][y]) if x != y else 0.0 for x in range(nd) for y in range(nd)])
+    order = (ctypes.c_int32 * nd)()
+    tp = (ctypes.c_double * nd)()
+    pb = ctypes.c_int32()
+    _check(lib().tqr_select_ndev(M, N, T, elem_size, nd, _times(times), sp, main_dev, order, tp, ctypes.byref(pb)),
+           None)
+    return list(order), list(tp), pb.value
 
 
 def tqr_generate_guide(rates):

@@ -104,3 +104,57 @@ def test_create_without_gpu_fails_cleanly(L):
         tqr.Plan(64, 128, 64, 16)
     assert e.value.status == 1
     assert L.tqr_destroy(None) == 0
+
+
+# ---------------------------------------------------------------- Alg. 2 / Alg. 3 + Eqs. 10-11
+from oracle import device_select as ds   # noqa: E402
+
+
+def test_select_main_pins(L):
+    """Alg. 2: among the devices that finish T before every other UE and E before
+    every other UT, the SLOWEST updater is the main device (the faster ones should update)."""
+    times = [(1, 1, 2, 2),     # speed 1/4, candidate
+             (1, 1, 1, 1),     # speed 1/2, candidate
+             (5, 5, 1, 1)]     # T = 5 > other UEs: not a candidate
+    assert tqr.tqr_select_main(times) == 0 == ds.main_selection(times)
+    # no candidate at all -> the fastest updater
+    times2 = [(9, 9, 3, 3), (9, 9, 1, 2), (9, 9, 2, 2)]
+    assert tqr.tqr_select_main(times2) == 1 == ds.main_selection(times2)
+    assert tqr.tqr_select_main([(1, 2, 3, 4)]) == 0
+
+
+def test_select_ndev_closed_form(L):
+    """Eq. 10 by hand: 4 identical devices, M = N = 8, (T, E, UT, UE) = (1, 2, 1, 2) s, free links.
+    p = 1: M(T+E) + 7 columns x M x (UT+UE) = 24 + 168 = 192.  p = 2 (guide {0,1}): main gets
+    columns 2,4,6 -> 24 + 72 = 96, device 1 gets 1,3,5,7 -> 96.  p = 4: main columns 4 -> 24 + 24 =
+    48, device 1 columns 1,5 -> 48.  Eq. 11 with 1 GB/s links, 8-byte elements, T = 1 adds
+    3 M (p - 1) 8 B / 1e9 + (M - 1) 8 B / 1e9 for p > 1."""
+    times = [(1.0, 2.0, 1.0, 2.0)] * 4
+    free = [[1e300] * 4 for _ in range(4)]
+    order, Tp, pb = tqr.tqr_select_ndev(8, 8, 1, 8, times, free, 0)
+    assert order == [0, 1, 2, 3]
+    np.testing.assert_allclose(Tp, [192.0, 96.0, 72.0, 48.0], rtol=1e-12)
+    assert pb == 4
+    slow = [[1e9] * 4 for _ in range(4)]
+    _, Tp2, _ = tqr.tqr_select_ndev(8, 8, 1, 8, times, slow, 0)
+    comm = [0.0] + [3 * 8 * (p - 1) * 8 / 1e9 + 7 * 8 / 1e9 for p in (2, 3, 4)]
+    np.testing.assert_allclose(Tp2, np.array([192.0, 96.0, 72.0, 48.0]) + comm, rtol=1e-12)
+    # links slow enough that one device wins
+    crawl = [[1.0] * 4 for _ in range(4)]
+    assert tqr.tqr_select_ndev(8, 8, 1, 8, times, crawl, 0)[2] == 1
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_select_matches_oracle(L, seed):
+    """Randomised heterogeneous devices: the library's Alg. 2/3 equal the step-by-step oracle."""
+    rng = np.random.default_rng(seed)
+    nd = int(rng.integers(1, 9))
+    times = [tuple(float(x) for x in rng.uniform(1e-4, 5e-3, 4)) for _ in range(nd)]
+    speed = rng.uniform(2e10, 9e11, (nd, nd)).tolist()
+    M, N, T = int(rng.integers(1, 70)), int(rng.integers(1, 70)), int(rng.choice([64, 256, 512]))
+    main = tqr.tqr_select_main(times)
+    assert main == ds.main_selection(times)
+    order, Tp, pb = tqr.tqr_select_ndev(M, N, T, 8, times, speed, main)
+    lo, Tpo, pbo = ds.num_dev_selection(M, N, T, 8, times, speed, main)
+    assert order == lo and pb == pbo
+    np.testing.assert_allclose(Tp, Tpo, rtol=1e-12)
