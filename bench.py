@@ -42,6 +42,9 @@ L2_BYTES = 126 * 2 ** 20
 SAMPLE_COLS = int(os.environ.get("TQR_ORACLE_SAMPLE_COLS", "2048"))
 
 
+METRIC = "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak"
+
+
 def flops(m, n):
     return 2.0 * m * n * n - 2.0 * n ** 3 / 3.0
 
@@ -163,11 +166,12 @@ def run_reference(args):
     m, n, nb, ib, seed = CONFIGS[args.config]
     value = statistics.median(vals)
     line = {
-        "impl": "reference", "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3)", "value": round(value, 3),
+        "impl": "reference", "metric": METRIC, "value": round(value, 3),
         "unit": "GFLOP/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(1e3 * statistics.median(times), 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
+                   "parallelism": "oracle on the host cores (rank 0 only)",
                    "sample": "first %d columns" % min(n, SAMPLE_COLS)},
         "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
                          "sample": desc},
@@ -369,7 +373,7 @@ def main():
                         "peak_source": peak_src, "launches_per_step": pcount // K,
                         "busy_ms_per_step": round(pms / K, 3), "share_of_step": round(pms / K / ms, 3)}
         line = {
-            "metric": "tiled QR GFLOP/s (2mn^2-2n^3/3) at 1/2/4/8 B200, % of FP64 tensor peak",
+            "metric": METRIC,
             "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
             "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",

@@ -78,6 +78,14 @@ typedef struct {
      * chains, then the group heads into head 0 by one chain (G - 1 + ceil(D/G) - 1 sequential
      * merges instead of D - 1). */
     int32_t tree_group;
+    /* Row split (NEXT-1 across devices; the paper's TT elimination P:L409-419 / TSQR): a single
+     * column tile (n <= nb) is split into ndev contiguous row blocks, one per owner (device or
+     * process); each owner factors its block (TS domains + merges), the owners' R factors are
+     * gathered to owner 0 (NCCL all-gather in multi-process mode) and merged there by one more
+     * factorisation of the stacked triu(R_g).  0 = auto (n <= nb, FP64, ndev > 1, >= 2 tiles per
+     * owner), 1 = force, -1 = off (column partition: owner(0) does all the work).  Row-split
+     * plans support tqr_factor / tqr_load / tqr_factor_tiles / tqr_store_r only. */
+    int32_t row_split;
 } tqr_options;
 
 /*

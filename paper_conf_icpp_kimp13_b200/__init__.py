@@ -34,7 +34,8 @@ class TqrError(RuntimeError):
 class Options(ctypes.Structure):
     _fields_ = [("logical_devices", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("nccl_id", ctypes.c_void_p), ("no_lookahead", ctypes.c_int32), ("profile", ctypes.c_int32),
-                ("tree_domain", ctypes.c_int32), ("tree_group", ctypes.c_int32)]
+                ("tree_domain", ctypes.c_int32), ("tree_group", ctypes.c_int32),
+                ("row_split", ctypes.c_int32)]
 
 
 class TileTimes(ctypes.Structure):
@@ -139,10 +140,10 @@ def _ptr_ld(x, rows: int, h=None):
 
 # ------------------------------------------------------------------ ABI-named functions
 def tqr_create(m, n, nb, ib, dtype=TQR_F64, ndev=1, guide=None, logical_devices=False, rank=0, world=1,
-               nccl_id=None, lookahead=True, profile=False, tree_domain=0, tree_group=0):
+               nccl_id=None, lookahead=True, profile=False, tree_domain=0, tree_group=0, row_split=0):
     g, glen = _i32_array(guide)
     opt = Options(int(bool(logical_devices)), int(rank), int(world), None, int(not lookahead), int(bool(profile)),
-                  int(tree_domain), int(tree_group))
+                  int(tree_domain), int(tree_group), int(row_split))
     idbuf = None
     if nccl_id is not None:
         idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128)

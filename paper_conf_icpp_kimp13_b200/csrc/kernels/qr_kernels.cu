@@ -443,6 +443,17 @@ __global__ void from_tiles_kernel(T* __restrict__ dst, int64_t lda, int64_t dst_
     }
 }
 
+// Row-split stage 2 input: the stacked R_g blocks (nb rows each, ld) keep only their upper
+// triangles: entry (r, c) with r % nb > c is zeroed (the reflectors stored below R_g's diagonal).
+template <class T>
+__global__ void zero_below_blocks_kernel(T* __restrict__ a, int64_t ld, int64_t rows, int64_t cols, int nb) {
+    const int64_t tot = rows * cols;
+    for (int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < tot; x += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t c = x / rows, r = x % rows;
+        if (r % nb > c) a[c * ld + r] = T(0);
+    }
+}
+
 // ============================================================================ launchers
 template <int NB, int IB, int W>
 static cudaError_t launch_panel_t(const PanelArgs& a, cudaStream_t s, int njobs) {
@@ -594,6 +605,16 @@ template cudaError_t launch_from_tiles<double>(double*, int64_t, int64_t, const 
                                                int64_t, int, int64_t, int64_t, int, cudaStream_t);
 template cudaError_t launch_from_tiles<float>(float*, int64_t, int64_t, const float*, const int32_t*, int,
                                               int64_t, int, int64_t, int64_t, int, cudaStream_t);
+
+template <class T>
+cudaError_t launch_zero_below_blocks(T* a, int64_t ld, int64_t rows, int64_t cols, int nb, cudaStream_t s) {
+    if (rows <= 0 || cols <= 0) return cudaSuccess;
+    const int grid = (int)std::min<int64_t>((rows * cols + 255) / 256, 148 * 8);
+    zero_below_blocks_kernel<T><<<grid, 256, 0, s>>>(a, ld, rows, cols, nb);
+    return cudaGetLastError();
+}
+template cudaError_t launch_zero_below_blocks<double>(double*, int64_t, int64_t, int64_t, int, cudaStream_t);
+template cudaError_t launch_zero_below_blocks<float>(float*, int64_t, int64_t, int64_t, int, cudaStream_t);
 
 size_t panel_smem_bytes(int nb, int ib) {
 #define TQR_PS(NB_, IB_) if (nb == NB_ && ib == IB_) return sizeof(Smem<NB_, IB_, IB_, true>);

@@ -134,6 +134,20 @@ struct tqr_plan_s {
     size_t bw_elems = 0;
     int64_t* dflag = nullptr;
 
+    // row split (tqr_options.row_split): per local owner a plan over its contiguous row block
+    // (kids), a stage-2 plan on owner 0 (top) factoring the stacked triu(R_g) (stk, G*nb x n)
+    bool rs = false;
+    std::vector<tqr_plan> kids;
+    std::vector<int> kid_owner, kid_dev;
+    std::vector<int64_t> rs_r0, rs_rows;    // per owner id
+    std::vector<void*> rs_zero;             // per kid: n x n zeros on its device
+    tqr_plan top = nullptr;
+    int top_dev = 0;
+    void* stk = nullptr;
+    void* rs_send = nullptr;
+    void* rs_recv = nullptr;
+    cudaStream_t rs_stream = nullptr;       // this process's gather stream
+
     bool nccl_mode = false;         // one process per GPU, panels broadcast with NCCL
     bool multiproc() const { return nccl_mode; }
     bool f32() const { return dtype == TQR_F32; }
@@ -380,6 +394,22 @@ tqr_status tqr_create(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dt
 
 tqr_status tqr_destroy(tqr_plan h) {
     if (!h) return TQR_OK;
+    if (h->rs) {
+        for (size_t i = 0; i < h->kids.size(); ++i) {
+            cudaSetDevice(h->kid_dev[i]);
+            tqr_destroy(h->kids[i]);
+            if (h->rs_zero[i]) cudaFree(h->rs_zero[i]);
+        }
+        if (h->top) { cudaSetDevice(h->top_dev); tqr_destroy(h->top); }
+        if (h->stk) cudaFree(h->stk);
+        if (h->rs_send) cudaFree(h->rs_send);
+        if (h->rs_recv) cudaFree(h->rs_recv);
+        if (h->rs_stream) cudaStreamDestroy(h->rs_stream);
+        if (h->comm && h->nccl) h->nccl->CommDestroy(h->comm);
+        cudaGetLastError();
+        delete h;
+        return TQR_OK;
+    }
     for (auto& o : h->owners) {
         cudaSetDevice(o.dev);
         if (o.s_panel) cudaStreamSynchronize(o.s_panel);
@@ -395,6 +425,83 @@ tqr_status tqr_destroy(tqr_plan h) {
     for (auto& o : h->owners) free_owner(o);
     cudaGetLastError();
     delete h;
+    return TQR_OK;
+}
+
+// Row-split plan (see tqr_options.row_split): owner g holds tile rows [g p / G, (g+1) p / G).
+static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
+                                   const tqr_options& o, bool use_nccl, int world, tqr_plan* out) {
+    const int64_t p = (m + nb - 1) / nb;
+    if (n > nb) return fail(nullptr, TQR_ERR_UNSUPPORTED, "row split: a single column tile (n <= nb) only");
+    tqr_plan h = new tqr_plan_s();
+    h->rs = true;
+    h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)p; h->q = 1;
+    h->dtype = dtype; h->ndev = ndev; h->es = (dtype == TQR_F32) ? 4 : 8;
+    h->guide.assign(1, 0);
+    h->owner_of.assign(1, 0);
+    h->rank = use_nccl ? o.rank : 0;
+    h->world = world;
+    h->nccl_mode = use_nccl;
+    h->profile = o.profile != 0;
+    auto bail = [&](tqr_status st) { std::string e = h->err; tqr_destroy(h); g_create_error = e; return st; };
+    for (int g = 0; g < ndev; ++g) {
+        const int64_t t0 = g * p / ndev, t1 = (g + 1) * p / ndev;
+        h->rs_r0.push_back(t0 * nb);
+        h->rs_rows.push_back(std::min<int64_t>(t1 * nb, m) - t0 * nb);
+        if (h->rs_rows.back() < n) return bail(fail(h, TQR_ERR_UNSUPPORTED, "row split: owner %d gets %lld < n rows", g, (long long)h->rs_rows.back()));
+    }
+    int cur = 0;
+    cudaGetDevice(&cur);
+    tqr_options co{};
+    co.logical_devices = 1;   // each kid lives on the current device when created
+    co.no_lookahead = o.no_lookahead;
+    co.profile = o.profile;
+    co.tree_domain = o.tree_domain;
+    co.tree_group = o.tree_group;
+    co.row_split = -1;
+    for (int g = 0; g < ndev; ++g) {
+        if (use_nccl && g != h->rank) continue;
+        const int dev = (use_nccl || o.logical_devices) ? cur : g;
+        if (cudaSetDevice(dev) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "cudaSetDevice(%d)", dev));
+        tqr_plan kid = nullptr;
+        tqr_status st = tqr_create_ex(h->rs_rows[g], n, nb, ib, dtype, 1, nullptr, 0, &co, &kid);
+        if (st) return bail(fail(h, st, "row split: owner %d plan: %s", g, g_create_error.c_str()));
+        h->kids.push_back(kid);
+        h->kid_owner.push_back(g);
+        h->kid_dev.push_back(dev);
+        void* z = nullptr;
+        if (cudaMalloc(&z, (size_t)h->es * n * n) != cudaSuccess || cudaMemset(z, 0, (size_t)h->es * n * n) != cudaSuccess)
+            return bail(fail(h, TQR_ERR_ALLOC, "row split: zero buffer"));
+        h->rs_zero.push_back(z);
+        if (g == 0) {
+            h->top_dev = dev;
+            tqr_options to = co;
+            to.tree_domain = -1;
+            st = tqr_create_ex((int64_t)ndev * nb, n, nb, ib, dtype, 1, nullptr, 0, &to, &h->top);
+            if (st) return bail(fail(h, st, "row split: stage-2 plan: %s", g_create_error.c_str()));
+            if (cudaMalloc(&h->stk, (size_t)h->es * ndev * nb * n) != cudaSuccess)
+                return bail(fail(h, TQR_ERR_ALLOC, "row split: stacked R buffer"));
+        }
+        if (use_nccl) {
+            if (cudaMalloc(&h->rs_send, (size_t)h->es * nb * n) != cudaSuccess ||
+                cudaMalloc(&h->rs_recv, (size_t)h->es * ndev * nb * n) != cudaSuccess)
+                return bail(fail(h, TQR_ERR_ALLOC, "row split: gather buffers"));
+        }
+    }
+    cudaSetDevice(use_nccl || o.logical_devices ? cur : 0);
+    if (cudaStreamCreateWithFlags(&h->rs_stream, cudaStreamNonBlocking) != cudaSuccess)
+        return bail(fail(h, TQR_ERR_CUDA, "row split: stream"));
+    if (use_nccl) {
+        const char* why = nullptr;
+        h->nccl = tqr::nccl_api(&why);
+        if (!h->nccl) return bail(fail(h, TQR_ERR_NCCL, "NCCL unavailable: %s", why));
+        ncclUniqueId id;
+        std::memcpy(&id, o.nccl_id, sizeof(id));
+        ncclResult_t r = h->nccl->CommInitRank(&h->comm, world, id, h->rank);
+        if (r != ncclSuccess) return bail(fail(h, TQR_ERR_NCCL, "ncclCommInitRank: %s", h->nccl->GetErrorString(r)));
+    }
+    cudaSetDevice(cur);
+    *out = h;
     return TQR_OK;
 }
 
@@ -425,6 +532,12 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     if (!use_nccl && !o.logical_devices && ndev > ndevices)
         return fail(nullptr, TQR_ERR_ARG, "ndev %d > %d visible CUDA devices (set logical_devices)", ndev, ndevices);
 
+    {
+        const int64_t pp = (m + nb - 1) / nb, qq = (n + nb - 1) / nb;
+        const bool rs = o.row_split > 0 ||
+                        (o.row_split == 0 && qq == 1 && ndev > 1 && dtype == TQR_F64 && pp >= 2 * ndev);
+        if (rs) return create_row_split(m, n, nb, ib, dtype, ndev, o, use_nccl, world, out);
+    }
     tqr_plan h = new tqr_plan_s();
     h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)((m + nb - 1) / nb); h->q = (int)((n + nb - 1) / nb);
     h->dtype = dtype; h->ndev = ndev; h->guide = g;
@@ -605,12 +718,32 @@ int32_t tqr_owner(tqr_plan h, int64_t j) {
 int64_t tqr_launch_count(tqr_plan h) {
     if (!h) return 0;
     int64_t c = h->launches;
+    for (auto k : h->kids) c += tqr_launch_count(k);
+    if (h->top) c += tqr_launch_count(h->top);
     h->launches = 0;
     return c;
 }
 
 tqr_status tqr_kernel_stats(tqr_plan h, int32_t which, int64_t* count, double* ms, double* flops, int32_t reset) {
     if (!h || which < 0 || which > 3) return fail(h, TQR_ERR_ARG, "kernel_stats: bad arguments");
+    if (h->rs) {   // the owners' row blocks run concurrently: count and flops add, time is the max
+        int64_t c = 0;
+        double t = 0.0, f = 0.0;
+        std::vector<tqr_plan> all(h->kids);
+        if (h->top) all.push_back(h->top);
+        for (size_t i = 0; i < all.size(); ++i) {
+            int64_t ci = 0;
+            double ti = 0.0, fi = 0.0;
+            tqr_kernel_stats(all[i], which, &ci, &ti, &fi, reset);
+            c += ci;
+            f += fi;
+            t = (all[i] == h->top) ? t + ti : std::max(t, ti);
+        }
+        if (count) *count = c;
+        if (ms) *ms = t;
+        if (flops) *flops = f;
+        return TQR_OK;
+    }
     if (count) *count = h->stats[which].count;
     if (ms) *ms = h->stats[which].ms;
     if (flops) *flops = h->stats[which].flops;
@@ -741,9 +874,97 @@ PanelRefs recv_refs(const tqr_plan_s*, Owner& O, int slot) {
 }
 }  // namespace
 
+// ------------------------------------------------------------------ row split (NEXT-1 across owners)
+namespace {
+tqr_status kid_fail(tqr_plan h, tqr_plan kid, tqr_status st) {
+    h->poisoned = h->poisoned || st == TQR_ERR_CUDA || st == TQR_ERR_NCCL;
+    return fail(h, st, "row split: %s", tqr_last_error(kid));
+}
+tqr_status rs_load(tqr_plan h, const void* A, int64_t lda) {
+    h->factored = false;
+    for (size_t i = 0; i < h->kids.size(); ++i) {
+        CUDA_TRY(h, cudaSetDevice(h->kid_dev[i]));
+        const int g = h->kid_owner[i];
+        tqr_status st = tqr_load(h->kids[i], static_cast<const char*>(A) + h->rs_r0[g] * h->es, lda);
+        if (st) return kid_fail(h, h->kids[i], st);
+    }
+    return TQR_OK;
+}
+// every owner factors its row block; the owners' R factors (tile 0 of each block) are stacked on
+// owner 0 (peer copies, or an NCCL all-gather) with their reflectors zeroed, and factored again
+tqr_status rs_factor(tqr_plan h) {
+    const int G = h->ndev, nb = h->nb;
+    const int64_t n = h->n, es = h->es, ld = (int64_t)G * nb;
+    for (size_t i = 0; i < h->kids.size(); ++i) {
+        CUDA_TRY(h, cudaSetDevice(h->kid_dev[i]));
+        tqr_status st = tqr_factor_tiles(h->kids[i]);
+        if (st) return kid_fail(h, h->kids[i], st);
+    }
+    if (h->multiproc()) {
+        tqr_plan kid = h->kids[0];
+        CUDA_TRY(h, cudaSetDevice(h->kid_dev[0]));
+        CUDA_TRY(h, cudaMemcpyAsync(h->rs_send, kid->owners[0].tiles, (size_t)es * nb * n, cudaMemcpyDeviceToDevice,
+                                    h->rs_stream));
+        const ncclDataType_t dt = h->f32() ? ncclFloat32 : ncclFloat64;
+        NCCL_TRY(h, h->nccl->AllGather(h->rs_send, h->rs_recv, (size_t)nb * n, dt, h->comm, h->rs_stream));
+        if (h->top) {
+            for (int g = 0; g < G; ++g)
+                CUDA_TRY(h, cudaMemcpy2DAsync(h->at(h->stk, (int64_t)g * nb), ld * es, h->at(h->rs_recv, (int64_t)g * nb * n),
+                                              nb * es, nb * es, n, cudaMemcpyDeviceToDevice, h->rs_stream));
+        }
+    } else {
+        CUDA_TRY(h, cudaSetDevice(h->top_dev));
+        for (size_t i = 0; i < h->kids.size(); ++i)
+            CUDA_TRY(h, cudaMemcpy2DAsync(h->at(h->stk, (int64_t)h->kid_owner[i] * nb), ld * es,
+                                          h->kids[i]->owners[0].tiles, nb * es, nb * es, n, cudaMemcpyDefault,
+                                          h->rs_stream));
+    }
+    if (h->top) {
+        CUDA_TRY(h, cudaSetDevice(h->top_dev));
+        if (h->f32()) CUDA_TRY(h, tqr::launch_zero_below_blocks<float>((float*)h->stk, ld, ld, n, nb, h->rs_stream));
+        else CUDA_TRY(h, tqr::launch_zero_below_blocks<double>((double*)h->stk, ld, ld, n, nb, h->rs_stream));
+        h->launches++;
+        CUDA_TRY(h, cudaStreamSynchronize(h->rs_stream));
+        tqr_status st = tqr_load(h->top, h->stk, ld);
+        if (!st) st = tqr_factor_tiles(h->top);
+        if (st) return kid_fail(h, h->top, st);
+    } else {
+        CUDA_TRY(h, cudaStreamSynchronize(h->rs_stream));
+    }
+    h->factored = true;
+    return TQR_OK;
+}
+// each owner writes its rows (R_g + zeros), then zeros over R_g; owner 0 writes the final R
+tqr_status rs_store(tqr_plan h, void* A, int64_t lda) {
+    const int64_t n = h->n, es = h->es, ld = (int64_t)h->ndev * h->nb;
+    for (size_t i = 0; i < h->kids.size(); ++i) {
+        CUDA_TRY(h, cudaSetDevice(h->kid_dev[i]));
+        const int g = h->kid_owner[i];
+        char* Ag = static_cast<char*>(A) + h->rs_r0[g] * es;
+        tqr_status st = tqr_store_r(h->kids[i], Ag, lda);
+        if (st) return kid_fail(h, h->kids[i], st);
+        if (g != 0) {
+            CUDA_TRY(h, cudaMemcpy2D(Ag, lda * es, h->rs_zero[i], n * es, n * es, n, cudaMemcpyDefault));
+        }
+    }
+    if (h->top) {
+        CUDA_TRY(h, cudaSetDevice(h->top_dev));
+        tqr_status st = tqr_store_r(h->top, h->stk, ld);
+        if (st) return kid_fail(h, h->top, st);
+        CUDA_TRY(h, cudaMemcpy2D(A, lda * es, h->stk, ld * es, n * es, n, cudaMemcpyDefault));
+    }
+    return TQR_OK;
+}
+}  // namespace
+
 // ------------------------------------------------------------------ a1: load
 tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
     if (!h) return TQR_ERR_ARG;
+    if (h->rs) {
+        if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+        if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "load: A is NULL or lda < m");
+        return rs_load(h, A, lda);
+    }
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "load: A is NULL or lda < m");
     const PtrInfo pi = classify(A);
@@ -868,6 +1089,7 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
 tqr_status tqr_factor_tiles(tqr_plan h) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (h->rs) return rs_factor(h);
     const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
     // bulk-update streams: round-robin (column lc on stream lc % S) for resident data; a streamed
     // factor maps contiguous chunks of columns to streams instead, so the early chunks run through
@@ -1086,6 +1308,7 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "store_r before factor");
     if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "store_r: A is NULL or lda < m");
+    if (h->rs) return rs_store(h, A, lda);
     const PtrInfo pi = classify(A);
     const int64_t nb = h->nb, es = h->es;
     { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
@@ -1121,6 +1344,12 @@ tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "factor: A is NULL or lda < m");
+    if (h->rs) {
+        tqr_status st = rs_load(h, A, lda);
+        if (!st) st = rs_factor(h);
+        if (!st) st = rs_store(h, A, lda);
+        return st;
+    }
     const PtrInfo pi = classify(A);
     bool resident = true;
     for (auto& o : h->owners)
@@ -1232,6 +1461,7 @@ tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nr
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "apply_qt before a successful factor");
     if (!(trans == 'T' || trans == 't' || trans == 'N' || trans == 'n')) return fail(h, TQR_ERR_ARG, "trans must be 'T' or 'N'");
+    if (h->rs) return fail(h, TQR_ERR_UNSUPPORTED, "apply_qt: row-split plans keep Q distributed (not supported)");
     if (nrhs < 0 || (nrhs > 0 && (!B || ldb < h->m))) return fail(h, TQR_ERR_ARG, "apply_qt: bad B/ldb/nrhs");
     if (nrhs == 0) return TQR_OK;
     int dev = 0;
@@ -1258,6 +1488,7 @@ tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "solve_ls before a successful factor");
     if (nrhs < 0 || (nrhs > 0 && (!B || ldb < h->m))) return fail(h, TQR_ERR_ARG, "solve_ls: bad B/ldb/nrhs");
+    if (h->rs) return fail(h, TQR_ERR_UNSUPPORTED, "solve_ls: row-split plans keep Q distributed (not supported)");
     if (nrhs == 0) return TQR_OK;
     int dev = 0;
     tqr_status st = single_device(h, &dev);
@@ -1327,6 +1558,7 @@ const NcclApi* nccl_api(const char** why) {
             api.CommDestroy = (decltype(api.CommDestroy))sym("ncclCommDestroy");
             api.CommGetAsyncError = (decltype(api.CommGetAsyncError))sym("ncclCommGetAsyncError");
             api.Broadcast = (decltype(api.Broadcast))sym("ncclBroadcast");
+            api.AllGather = (decltype(api.AllGather))sym("ncclAllGather");
             api.GroupStart = (decltype(api.GroupStart))sym("ncclGroupStart");
             api.GroupEnd = (decltype(api.GroupEnd))sym("ncclGroupEnd");
             api.GetErrorString = (decltype(api.GetErrorString))sym("ncclGetErrorString");

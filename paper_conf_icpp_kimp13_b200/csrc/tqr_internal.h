@@ -92,6 +92,9 @@ template <class T>
 cudaError_t launch_from_tiles(T* dst, int64_t lda, int64_t dst_group_stride, const T* src, const int32_t* cols_dev,
                               int ncols, int64_t src_col_stride, int nb, int64_t m_rows, int64_t n_valid,
                               int local_dst, cudaStream_t s);
+// zero (r, c) with r % nb > c in a rows x cols column-major block stack (ld)
+template <class T>
+cudaError_t launch_zero_below_blocks(T* a, int64_t ld, int64_t rows, int64_t cols, int nb, cudaStream_t s);
 // Step i of the tile back substitution (trsm.cu): X_i = R_ii^-1 C_i, then C_r -= R_ri X_i, r < i.
 // Rcol = column tile i of R in tile storage (tile r at Rcol + r*nb*nb); C = mp x 32*nslices, ld ldc.
 template <class T>

@@ -376,6 +376,54 @@ def test_nccl_transport_single_rank_bitwise():
     assert e.value.status == 7
 
 
+@pytest.mark.parametrize("m,n,nb,ib,ndev", [
+    (8192, 512, 512, 32, 2),      # 16 tiles -> 8 + 8 rows tiles, each owner's block a TS tree
+    (12800, 512, 512, 32, 3),     # 25 tiles -> 8 / 8 / 9
+    (5000, 200, 256, 32, 4),      # ragged: n < nb, m not a multiple of nb
+    (4096, 64, 64, 16, 8),        # 64 tiles over 8 owners
+])
+def test_row_split_matches_oracle(m, n, nb, ib, ndev):
+    """Row split (NEXT-1 across owners, TSQR): each logical owner factors its contiguous row
+    block, the owners' R factors are stacked on owner 0 and factored again.  R is unique, so it
+    must match the oracle like the single-owner tree; every entry below R is zero."""
+    A = synthetic.gaussian(m, n, 7500 + m + ndev)
+    plan = tqr.Plan(m, n, nb, ib, ndev=ndev, logical_devices=True, row_split=1)
+    Ad = dev_colmajor(A)
+    plan.factor(Ad)
+    Rg = to_np(Ad)
+    ref = oracle.qr(A)
+    assert colnorm_rel_err(np.triu(Rg[:n]), ref.R) <= R_TOL
+    assert np.all(np.tril(Rg, -1) == 0.0) and np.all(Rg[n:] == 0.0)
+    _, R1 = gpu_qr(A, nb, ib)                               # single owner
+    assert colnorm_rel_err(np.triu(Rg[:n]), np.triu(R1[:n])) <= R_TOL
+    Ah = np.asfortranarray(A.copy())                       # host A, three-phase ABI path
+    plan.load(Ah)
+    plan.factor_tiles()
+    Rh = np.zeros((n, m)).T
+    Rh = np.asfortranarray(np.full((m, n), 3.0))
+    plan.store_r(Rh)
+    assert np.array_equal(Rh, Rg)
+    with pytest.raises(tqr.TqrError) as e:
+        plan.apply_qt(dev_colmajor(np.ones((m, 1))))
+    assert e.value.status == 7
+    plan.close()
+
+
+def test_row_split_nccl_single_rank():
+    """The multi-process row split (NCCL all-gather of the owners' R factors) with a 1-rank
+    communicator: one row block, then the stage-2 refactorisation of its R."""
+    m, n, nb, ib = 8192, 512, 512, 32
+    A = synthetic.gaussian(m, n, 7600)
+    uid = tqr.tqr_nccl_unique_id()
+    plan = tqr.Plan(m, n, nb, ib, ndev=1, rank=0, world=1, nccl_id=uid, row_split=1)
+    Ad = dev_colmajor(A)
+    plan.factor(Ad)
+    Rg = to_np(Ad)
+    assert colnorm_rel_err(np.triu(Rg[:n]), oracle.qr(A).R) <= R_TOL
+    assert np.all(np.tril(Rg, -1) == 0.0)
+    plan.close()
+
+
 def _sampled_checks(plan, Ad, Rd, m, n, nb, seed, ncols_oracle):
     """Full-size parity in the bench launch configuration (tqr_load + tqr_factor_tiles +
     tqr_store_r on device buffers):

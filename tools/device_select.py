@@ -55,6 +55,7 @@ def tile_times(nb, ib):
         t_load = timed(lambda: plan.load(A0))
         tp[p] = t_all - t_load
         if p == 16:
+            f()
             B0 = torch.randn((18 * nb, m), dtype=torch.float64, device="cuda", generator=g).t()
             B = B0.clone()
             t_app = timed(lambda: plan.apply_qt(B, "T"))
