@@ -380,7 +380,9 @@ def main():
             ("pct_fp32_ffma_peak" if f32 else "pct_fp64_peak"): round(100.0 * value / 1e3 / (peak * world), 2),
             "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
                        "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": list(range(world)),
-                       "parallelism": "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
+                       "parallelism": ("row-split x%d (per-rank TS trees + NCCL all-gather of the R factors, "
+                                       "stage-2 merge on rank 0)" % world) if (n <= nb and world > 1) else
+                                      "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
                        "tree": args.tree, "tree_group": args.tree_group,
                        "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (es * m * n / 2 ** 30)
                        if es * m * n > L2_BYTES else "input fits L2 (no flush)"},
