@@ -8,10 +8,12 @@ metric : tiled QR GFLOP/s = (2mn^2 - 2n^3/3) / t, whole job, plus % of the FP64 
 step   : one pass of the whole hot path over the config's matrix:
          tqr_load (col-major -> tiles) + tqr_factor_tiles (GEQRT/TSQRT panels, UNMQR/TSMQR
          updates, lookahead, broadcasts) + tqr_store_r (R out).  Input resident in HBM.
-e2e    : the same through tqr_factor-equivalent calls on PINNED HOST buffers (H2D of A and
-         D2H of R inside the timed region).
-N > 1  : launched by torchrun; one process per GPU, column tiles partitioned by the guide
-         array {0..N-1} (Eq. 12), panels broadcast with NCCL.  Strong scaling (same matrix).
+e2e    : the same through tqr_factor on a PINNED HOST A (H2D of A and D2H of R inside the
+         timed region, pipelined with the factorization by the library).
+N > 1  : launched by torchrun; one process per GPU, column tiles partitioned by a guide array
+         (Eq. 12; --guide: cyclic {0..N-1}, or pairs {0,0,1,1,..} -- default for N >= 8), panels
+         broadcast with NCCL; a single column tile (C4) is split by rows instead (row split).
+         Strong scaling (same matrix).
 --impl reference : the CPU oracle (Algorithm 1, oracle/) timed on this host's cores on a
          bounded sample of the same workload (first 2048 columns of the config's matrix).
 """
@@ -196,6 +198,10 @@ def main():
     ap.add_argument("--no-lookahead", action="store_true")
     ap.add_argument("--tree", type=int, default=0,
                     help="elimination tree: 0 auto (tree for q == 1), -1 flat TS, L > 0 TS domains of L tiles")
+    ap.add_argument("--guide", default="auto", choices=["auto", "cyclic", "pairs"],
+                    help="N > 1 column distribution (Eq. 12 guide array): cyclic {0..N-1}; pairs "
+                         "{0,0,1,1,..}: the lookahead column is local every other step; auto = pairs "
+                         "for N >= 8 (critical-path bound), cyclic otherwise")
     ap.add_argument("--solve", type=int, default=0,
                     help="also time tqr_solve_ls with this many right-hand sides (NEXT-3; 'solve' key)")
     ap.add_argument("--tree-group", type=int, default=0,
@@ -233,7 +239,10 @@ def main():
         obj = [tqr.tqr_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
-    plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, rank=rank, world=world, nccl_id=nccl_id,
+    gmode = args.guide if args.guide != "auto" else ("pairs" if world >= 8 else "cyclic")
+    guide = [d for d in range(world) for _ in range(2 if gmode == "pairs" else 1)]
+    plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, guide=guide,
+                    rank=rank, world=world, nccl_id=nccl_id,
                     lookahead=not args.no_lookahead, profile=True, tree_domain=args.tree,
                     tree_group=args.tree_group)
 
@@ -379,7 +388,7 @@ def main():
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             ("pct_fp32_ffma_peak" if f32 else "pct_fp64_peak"): round(100.0 * value / 1e3 / (peak * world), 2),
             "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
-                       "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": list(range(world)),
+                       "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": guide,
                        "parallelism": ("row-split x%d (per-rank TS trees + NCCL all-gather of the R factors, "
                                        "stage-2 merge on rank 0)" % world) if (n <= nb and world > 1) else
                                       "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,

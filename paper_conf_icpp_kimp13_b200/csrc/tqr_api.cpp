@@ -115,6 +115,8 @@ struct tqr_plan_s {
     size_t prog_n = 0;
     bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
     bool streamed = false;
+    bool cp_probe = false;          // TQR_CRITICAL_PATH_PROBE=1 (diagnostic, wrong results): skip the
+                                    // bulk updates -> panels + lookahead only = the critical path
     void* sA = nullptr;
     int64_t slda = 0;
     int ngroups(int D) const { return (tree_G > 1 && D > tree_G) ? (D + tree_G - 1) / tree_G : 1; }
@@ -550,6 +552,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_LA_OVERLAP")) h->la_overlap = atoi(e) != 0;
+    if (const char* e = getenv("TQR_CRITICAL_PATH_PROBE")) h->cp_probe = atoi(e) != 0;
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
     // Tree mode (NEXT-1): TS domains of L tiles factored one per CTA, merged by a flat TT chain.
     // Auto: a single panel column (q == 1, e.g. C4) whose flat chain has parallelism 1.
@@ -1216,7 +1219,8 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 // owner: the update runs beside PANEL(k) (already enqueued, so its CTAs are
                 // dispatched first) and waits per reflector tile on the panel's flags; otherwise it
                 // follows the whole panel (or the broadcast) on the panel stream.
-                const bool ovl = mine && h->la_overlap && !h->f32() && h->ndom(k) == 1;
+                // (not with logical owners: several owners' lookaheads could then spin on one GPU)
+                const bool ovl = mine && h->la_overlap && !h->logical && !h->f32() && h->ndom(k) == 1;
                 cudaStream_t sl = ovl ? D.s_look : D.s_panel;
                 if (!ovl) CUDA_TRY(h, cudaStreamWaitEvent(sl, ready, 0));
                 if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_u[stream_of(first, (int)D.cols.size())][k - 1], 0));
@@ -1246,7 +1250,9 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     gs = S;
                 }
                 cudaStream_t su = D.s_u[uu];
-                if (ng > 0) {
+                if (h->cp_probe && ng > 0) {   // keep the dependency structure, skip the work
+                    CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
+                } else if (ng > 0) {
                     CUDA_TRY(h, cudaStreamWaitEvent(su, ready, 0));
                     if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[uu][k], su));
                     const int wb = w_bulk(h);
