@@ -315,8 +315,9 @@ def main():
         ems = max_over_ranks(tot / ke)
         e2e = {"value": round(fl / (ems * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
                "ms_per_step": round(ems, 3), "h2d_bytes_per_step": es * m * n, "d2h_bytes_per_step": es * m * n,
-               "api": "tqr_factor(pinned host A): per-column H2D + layout convert, factorization and per-column "
-                      "R-out + D2H overlapped inside the call"}
+               "api": "tqr_factor(pinned host A): H2D + layout convert and R-out + D2H pipelined with the "
+                      "factorization inside the call (per column tile; per row chunk of TS domains for a "
+                      "single tile column)"}
         del Ah
 
     # ---- least squares throughput (NEXT-3): Q^T B (update kernel) + tile back substitution on a

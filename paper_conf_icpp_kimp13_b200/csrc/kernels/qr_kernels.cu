@@ -194,7 +194,7 @@ __global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
     using G = Geom<NB, IB, IB>;
     constexpr int NBLK = NB / IB;
     const int64_t tile = (int64_t)NB * NB;
-    const int head = a.k + blockIdx.x * a.L;
+    const int head = a.k + (a.dom0 + (int)blockIdx.x) * a.L;
     const int end = min(head + a.L, a.p);
     double* Ah = a.col + (int64_t)head * tile;
     double* himg = (head == a.k) ? a.Vexp : a.Vimg + (int64_t)head * tile;

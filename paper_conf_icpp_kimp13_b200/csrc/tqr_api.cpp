@@ -72,6 +72,7 @@ struct Owner {
     cudaStream_t s_io = nullptr;                    // streamed tqr_factor: per-column H2D + a1, a8 + D2H
     cudaStream_t s_look = nullptr;                  // lookahead update overlapped with its own panel
     std::vector<cudaEvent_t> ev_load;               // ev_load[lc]: local column lc resident in tile layout
+    std::vector<cudaEvent_t> ev_chunk, ev_dom;      // streamed tall factor: row chunk c loaded / its domains done
     std::vector<cudaStream_t> s_u;                  // bulk-update streams (column lc -> s_u[lc % S])
     std::vector<cudaEvent_t> ev_panel, ev_recv, ev_look;
     std::vector<std::vector<cudaEvent_t>> ev_u;     // ev_u[u][k]: stream u finished its step-k updates
@@ -115,6 +116,7 @@ struct tqr_plan_s {
     size_t prog_n = 0;
     bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
     bool streamed = false;
+    bool domains_done = false;      // streamed tall factor: the TS domains were launched per row chunk
     bool cp_probe = false;          // TQR_CRITICAL_PATH_PROBE=1 (diagnostic, wrong results): skip the
                                     // bulk updates -> panels + lookahead only = the critical path
     void* sA = nullptr;
@@ -219,7 +221,7 @@ void free_owner(Owner& o) {
     F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp); F(o.Mimg); F(o.MT); F(o.Mt);
     for (int s = 0; s < 2; ++s) { F(o.rb_M[s]); F(o.rb_MT[s]); }
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
-    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref, &o.ev_load})
+    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref, &o.ev_load, &o.ev_chunk, &o.ev_dom})
         for (auto e : *v) if (e) cudaEventDestroy(e);
     for (auto* vv : {&o.ev_u, &o.tm0, &o.tm1})
         for (auto& v : *vv) for (auto e : v) if (e) cudaEventDestroy(e);
@@ -1037,7 +1039,9 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
         }
         // tree: D TS domains (one CTA each), then the flat merge chain of the domain heads' R
         // factors against head 0 (the panel kernel in TSQRT-only mode on the merge bottoms)
-        if (h->tree_one_cta) {
+        if (h->domains_done) {
+            // launched per row chunk by the streamed tall factor; the panel stream waited for them
+        } else if (h->tree_one_cta) {
             tqr::DomainArgs da{a.col, a.T, a.Vimg, a.Vexp, k, p, h->tree_L};
             CUDA_TRY(h, tqr::launch_domains(nb, ib, da, D, O.s_panel));
         } else {
@@ -1341,6 +1345,83 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
     return sync_all(h);
 }
 
+// Streamed factor of a single tile column in tree mode (C4-like, one owner, one CTA per domain):
+// the rows arrive in NC chunks of whole TS domains on the I/O stream (H2D + a1 per chunk); each
+// chunk's domains start on their own stream as soon as the chunk is resident; the rows >= nb of a
+// chunk are zero in the result, so they are written back (zeros, device -> host on the comm
+// stream, full duplex with the loads) as soon as the chunk has been read; after the merges only
+// the first tile row (R) is copied out.
+namespace {
+tqr_status factor_streamed_tall(tqr_plan h, void* A, int64_t lda) {
+    Owner& O = h->owners[0];
+    const int nb = h->nb, p = h->p, L = h->tree_L, D = h->ndom(0);
+    const int64_t m = h->m, es = h->es, tile = (int64_t)nb * nb, colsz = (int64_t)p * tile;
+    const int NC = std::min(D, 8);
+    CUDA_TRY(h, cudaSetDevice(O.dev));
+    tqr_status st = ensure_io(h, O);
+    if (st) return st;
+    auto mk = [&](std::vector<cudaEvent_t>& v) -> tqr_status {
+        while ((int)v.size() < NC) {
+            cudaEvent_t e;
+            CUDA_TRY(h, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+            v.push_back(e);
+        }
+        return TQR_OK;
+    };
+    if ((st = mk(O.ev_chunk)) || (st = mk(O.ev_dom))) return st;
+    const unsigned epoch0 = h->epoch;
+    h->epoch += 2;
+    h->factored = false;
+    double* col = h->at<double>(O.tiles, 0);
+    const PanelRefs r = own_refs(h, O, 0);
+    for (int c = 0; c < NC; ++c) {
+        const int d0 = (int)((int64_t)c * D / NC), d1 = (int)((int64_t)(c + 1) * D / NC);
+        const int t0 = d0 * L, t1 = std::min(d1 * L, p);
+        const int64_t r0 = (int64_t)t0 * nb, r1 = std::min<int64_t>((int64_t)t1 * nb, m);
+        void* slab = h->at(O.io, r0);
+        if (r1 > r0) {
+            CUDA_TRY(h, cudaMemcpy2DAsync(slab, m * es, static_cast<const char*>(A) + r0 * es, lda * es, (r1 - r0) * es,
+                                          h->n, cudaMemcpyDefault, O.s_io));
+        }
+        CUDA_TRY(h, tqr::launch_to_tiles<double>((const double*)slab, m, m * nb, col + (int64_t)t0 * tile, O.cols_dev,
+                                                 1, 1, colsz, nb, t1 - t0, std::max<int64_t>(r1 - r0, 0), h->n, O.s_io));
+        CUDA_TRY(h, cudaEventRecord(O.ev_chunk[c], O.s_io));
+        cudaStream_t sd = O.s_u[c % O.s_u.size()];
+        CUDA_TRY(h, cudaStreamWaitEvent(sd, O.ev_chunk[c], 0));
+        tqr::DomainArgs da{col, (double*)r.T, (double*)r.V, (double*)r.Vexp, 0, p, L};
+        da.dom0 = d0;
+        CUDA_TRY(h, tqr::launch_domains(nb, h->ib, da, d1 - d0, sd));
+        CUDA_TRY(h, cudaEventRecord(O.ev_dom[c], sd));
+        // result rows [max(r0, nb), r1) are zero: the slab rows were consumed by a1 -> zero them
+        // on the device and write them back while later chunks load
+        const int64_t z0 = std::max<int64_t>(r0, nb);
+        if (r1 > z0) {
+            CUDA_TRY(h, cudaStreamWaitEvent(O.s_comm, O.ev_chunk[c], 0));
+            void* zs = h->at(O.io, z0);
+            CUDA_TRY(h, cudaMemset2DAsync(zs, m * es, 0, (r1 - z0) * es, h->n, O.s_comm));
+            CUDA_TRY(h, cudaMemcpy2DAsync(static_cast<char*>(A) + z0 * es, lda * es, zs, m * es, (r1 - z0) * es, h->n,
+                                          cudaMemcpyDefault, O.s_comm));
+        }
+        h->launches += 2;
+    }
+    for (int c = 0; c < NC; ++c) CUDA_TRY(h, cudaStreamWaitEvent(O.s_panel, O.ev_dom[c], 0));
+    h->domains_done = true;
+    st = launch_panel_step(h, O, 0, epoch0 + 1);
+    h->domains_done = false;
+    if (st) return st;
+    // R: the first tile row only (a8 for rows 0..min(nb, m)), after the merges
+    const int64_t rr = std::min<int64_t>(nb, m);
+    CUDA_TRY(h, tqr::launch_from_tiles<double>((double*)O.io, m, m * nb, col, O.cols_dev, 1, colsz, nb, rr, h->n, 1,
+                                               O.s_panel));
+    CUDA_TRY(h, cudaMemcpy2DAsync(A, lda * es, O.io, m * es, rr * es, h->n, cudaMemcpyDefault, O.s_panel));
+    h->launches++;
+    st = sync_all(h);
+    if (st) return st;
+    h->factored = true;
+    return TQR_OK;
+}
+}  // namespace
+
 // A not resident on the owners' devices (host memory, or another GPU): the I/O is pipelined with
 // the factorization -- column tile j is copied in and converted (a1) on the owner's I/O stream,
 // PANEL(j) and the step-0 update of column j wait only for column j, and R of column k (a8) is
@@ -1370,6 +1451,9 @@ tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
     const int64_t nb = h->nb, es = h->es, colsz = (int64_t)h->p * nb * nb;
     h->factored = false;
     { tqr_status st0 = sync_entry(h, pi); if (st0) return st0; }
+    if (h->q == 1 && h->tree_L > 0 && h->tree_one_cta && h->owners.size() == 1 && !h->multiproc() && !h->f32() &&
+        h->ndom(0) > 1 && !getenv("TQR_NO_STREAMED_TALL"))
+        return factor_streamed_tall(h, A, lda);
     for (auto& o : h->owners) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, cudaSetDevice(o.dev));

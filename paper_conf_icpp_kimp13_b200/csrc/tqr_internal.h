@@ -37,6 +37,7 @@ struct DomainArgs {
     double* Vimg;
     double* Vexp;
     int k, p, L;
+    int dom0 = 0;      // first domain of this launch (CTA x factors domain dom0 + x)
 };
 cudaError_t launch_domains(int nb, int ib, const DomainArgs& a, int ndom, cudaStream_t s);
 // merge inputs: Mt[e] = triu(tile k + e*L) (zeros below the diagonal), e = 1..ndom-1

@@ -244,6 +244,26 @@ def test_streamed_host_factor_bitwise(m, n, nb, ib, kw, monkeypatch):
     plan.close()
 
 
+@pytest.mark.parametrize("m,n,nb,ib", [(8192, 512, 512, 32), (5000, 300, 512, 32), (24576, 256, 256, 32)])
+def test_streamed_tall_factor_bitwise(m, n, nb, ib, monkeypatch):
+    """Single tile column, tree mode with one CTA per domain: tqr_factor on a host A loads the rows
+    in chunks of whole domains, starts each chunk's domains as it lands, writes the zero rows back
+    early and R (first tile row) after the merges -- bitwise the device-resident result."""
+    monkeypatch.setenv("TQR_TREE_ONE_CTA", "1")
+    A = synthetic.gaussian(m, n, 7700 + m + n)
+    _, Rd = gpu_qr(A, nb, ib)
+    plan = tqr.Plan(m, n, nb, ib)
+    Ap = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    plan.factor(Ap)
+    assert np.array_equal(Ap.numpy(), Rd)
+    Ah = np.full((m + 5, n), 9.0, order="F")              # pageable, lda > m: rows m.. untouched
+    Ah[:m] = A
+    assert tqr.lib().tqr_factor(plan.h, Ah.ctypes.data, m + 5) == 0
+    assert np.array_equal(Ah[:m], Rd) and np.all(Ah[m:] == 9.0)
+    assert colnorm_rel_err(np.triu(Rd[:n]), oracle.qr(A).R) <= R_TOL
+    plan.close()
+
+
 @pytest.mark.parametrize("ndev,guide", [(2, None), (2, [1, 0]), (3, [1, 0, 1, 0, 1, 2]), (4, [0, 0, 1, 3, 2])])
 def test_logical_devices_partition_bitwise(ndev, guide):
     """Guide-array partitions (Eq. 12) on logical devices: identical R to the 1-owner run."""
