@@ -1261,12 +1261,12 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tm0[uu][k], su));
                     const int wb = w_bulk(h);
                     if (k == 0 && h->streamed) {
-                        // step 0 of a streamed factor: one launch per column, each after its load
-                        for (int c = g0; c < g0 + ng * gs; c += gs) {
-                            CUDA_TRY(h, cudaStreamWaitEvent(su, D.ev_load[c], 0));
-                            CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, c, gs, k, wb, nb / wb, true, su,
-                                               &h->launches));
-                        }
+                        // step 0 of a streamed factor: the chunk's columns load in order, so waiting
+                        // for its last one covers them all; one launch keeps the chunk's columns
+                        // concurrent (per-column launches on one stream would run one at a time)
+                        CUDA_TRY(h, cudaStreamWaitEvent(su, D.ev_load[g0 + (ng - 1) * gs], 0));
+                        CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, gs, k, wb, ng * (nb / wb), true, su,
+                                           &h->launches));
                     } else {
                         CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, gs, k, wb, ng * (nb / wb), true, su,
                                            &h->launches));
