@@ -298,12 +298,19 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     // wavefront apply (nsteps > 1): CTA = (step offset st, slice); step k = a.k +- st with its own
     // reflector column (V, T, Vexp + k * column strides); tile i of step k waits until the
     // previous step's CTA of the same slice has finished tile i (progress flags, lower CTA index)
+    // tree jobs (domL > 0): CTA = (job d, slice); job d is the chain of row tiles
+    // [k + d*domL, min(k + (d+1)*domL, p)) against its own head (the TS domains of a tree panel,
+    // or the level-1 merge groups over merge slots) -- independent row ranges, one launch
+    const bool jobs = a.domL > 0;
     const int st = a.nsteps > 1 ? (int)(blockIdx.x / a.nslc) : 0;
-    const int bid = a.nsteps > 1 ? (int)(blockIdx.x % a.nslc) : (int)blockIdx.x;
-    const int k = TRANS ? a.k + st : a.k - st;
+    const int jd = jobs ? (int)(blockIdx.x / a.nslc) : 0;
+    const int bid = (a.nsteps > 1 || jobs) ? (int)(blockIdx.x % a.nslc) : (int)blockIdx.x;
+    const int k = jobs ? a.k + jd * a.domL : (TRANS ? a.k + st : a.k - st);
+    const int pend = jobs ? min(k + a.domL, a.p) : a.p;
     const double* __restrict__ Vb = a.V + (int64_t)st * (TRANS ? 1 : -1) * a.vcol;
     const double* __restrict__ Tb = a.T + (int64_t)st * (TRANS ? 1 : -1) * a.tcol;
-    const double* __restrict__ Eb = a.Vexp + (int64_t)st * (TRANS ? 1 : -1) * a.ecol;
+    const double* __restrict__ Eb = (jobs && jd > 0) ? a.V + (int64_t)k * a.vstride * NB * NB
+                                                     : a.Vexp + (int64_t)st * (TRANS ? 1 : -1) * a.ecol;
     const int grp = bid / SPG;
     const int c0 = (bid % SPG) * W;
     double* Xg = a.X + (int64_t)(a.group0 + grp * a.gstride) * a.col_stride + (int64_t)c0 * a.ld;
@@ -316,10 +323,10 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
     // Reflector blocks in application order; block q of the sequence is staged (cp.async) while
     // block q-1's GEMM2 runs.  Forward: UNMQR blocks 0..NBLK-1, then for i = k+1..p-1 blocks
     // 0..NBLK-1 of V_i.  Backward: i = p-1..k+1 blocks NBLK-1..0, then UNMQR blocks NBLK-1..0.
-    const int ntiles = a.p - k - 1 + (a.do_unmqr ? 1 : 0);
+    const int ntiles = pend - k - 1 + (a.do_unmqr ? 1 : 0);
     auto tile_of = [&](int q) -> int {            // q-th tile of the sequence; -1 = UNMQR (row tile k)
         if (TRANS) return a.do_unmqr ? (q == 0 ? -1 : k + q) : k + 1 + q;
-        return (q < a.p - k - 1) ? a.p - 1 - q : -1;
+        return (q < pend - k - 1) ? pend - 1 - q : -1;
     };
     auto vblock = [&](int ti, int s) -> const double* {
         return (ti < 0 ? Eb : Vb + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;

@@ -790,7 +790,7 @@ struct PanelRefs {
 cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const void* Vexp, void* X, int64_t col_stride,
                     int64_t tile_stride, int64_t ld, int group0, int gstride, int k_head, int p_end, int do_unmqr,
                     int w, int nslices, bool trans, cudaStream_t s, int vstride = 1,
-                    const unsigned* wflags = nullptr, unsigned wepoch = 0) {
+                    const unsigned* wflags = nullptr, unsigned wepoch = 0, int domL = 0, int njobs = 1) {
     if (h->f32()) {
         tqr::UpdateArgsT<float> u;
         u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
@@ -803,7 +803,8 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
     u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
     u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr; u.vstride = vstride;
     u.wflags = wflags; u.wepoch = wepoch;
-    return tqr::launch_update(h->nb, h->ib, w, u, nslices, trans, s);
+    if (domL > 0) { u.domL = domL; u.nslc = nslices; }
+    return tqr::launch_update(h->nb, h->ib, w, u, nslices * njobs, trans, s);
 }
 // Q_k^T (trans) or Q_k applied to X.  Flat: one launch (UNMQR(k) + TSMQR(k+1..p-1)).  Tree (D > 1
 // domains of L tiles): per domain d, UNMQR of its head k + d*L and TSMQR of its tiles against the
@@ -821,11 +822,10 @@ cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col
         return update1(h, r.V, r.T, r.Vexp, X, col_stride, tile_stride, ld, group0, gstride, k, h->p, 1, w, nslices,
                        trans, s, 1, wflags, wepoch);
     }
-    auto dom = [&](int d) {
-        const int head = k + d * L, end = std::min(head + L, h->p);
-        const void* vex = d == 0 ? r.Vexp : h->at(r.V, (int64_t)head * h->vt);
-        return update1(h, r.V, r.T, vex, X, col_stride, tile_stride, ld, group0, gstride, head, end, 1, w, nslices,
-                       trans, s);
+    // all D domains in one launch (independent row ranges; job d = domain d, head k + d*L)
+    auto doms = [&]() {
+        return update1(h, r.V, r.T, r.Vexp, X, col_stride, tile_stride, ld, group0, gstride, k, h->p, 1, w, nslices,
+                       trans, s, 1, nullptr, 0, L, D);
     };
     const int NG = h->ngroups(D), G = h->tree_G;
     const int64_t tsz = (int64_t)h->ib * h->nb;
@@ -833,25 +833,24 @@ cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col
         return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L, ld, group0,
                        gstride, 0, D, 0, w, nslices, trans, s);
     };
-    auto grp = [&](int g) {   // level 1: group g's chain against its head gG
-        const int h0 = g * G, len = std::min(G, D - h0);
-        if (len < 2) return cudaSuccess;
-        return update1(h, h->at(r.M, (int64_t)h0 * h->vt), h->at(r.MT, (int64_t)h0 * tsz), r.M,
-                       h->at(X, (int64_t)(k + h0 * L) * tile_stride), col_stride, tile_stride * L, ld, group0, gstride,
-                       0, len, 0, w, nslices, trans, s);
+    // level 1: every group's chain against its head gG in one launch (jobs of G merge slots)
+    auto grps = [&]() {
+        (void)tsz;
+        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L, ld, group0,
+                       gstride, 0, D, 0, w, nslices, trans, s, 1, nullptr, 0, G, NG);
     };
     auto top = [&]() {   // level 2: group heads G, 2G, .. against head 0 (merge slots stride G)
         return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L * G, ld,
                        group0, gstride, 0, NG, 0, w, nslices, trans, s, G);
     };
-    if (nl) *nl += D + (NG > 1 ? NG + 1 : 1);
+    if (nl) *nl += (NG > 1 ? 3 : 2);
     cudaError_t e = cudaSuccess;
     if (trans) {
-        for (int d = 0; d < D && e == cudaSuccess; ++d) e = dom(d);
+        e = doms();
         if (NG == 1) {
             if (e == cudaSuccess) e = mrg();
         } else {
-            for (int g = 0; g < NG && e == cudaSuccess; ++g) e = grp(g);
+            if (e == cudaSuccess) e = grps();
             if (e == cudaSuccess) e = top();
         }
     } else {
@@ -859,9 +858,9 @@ cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col
             e = mrg();
         } else {
             e = top();
-            for (int g = NG - 1; g >= 0 && e == cudaSuccess; --g) e = grp(g);
+            if (e == cudaSuccess) e = grps();
         }
-        for (int d = D - 1; d >= 0 && e == cudaSuccess; --d) e = dom(d);
+        if (e == cudaSuccess) e = doms();
     }
     return e;
 }

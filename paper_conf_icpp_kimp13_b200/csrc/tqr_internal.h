@@ -70,7 +70,8 @@ struct UpdateArgsT {
     // step k +- st (TRANS: +) with V, T, Vexp advanced by st * (vcol, tcol, ecol) elements; prog
     // (nsteps * nslc, zeroed) counts the chain tiles each CTA has finished
     int nsteps = 1;
-    int nslc = 0;
+    int nslc = 0;                        // slices per step (nsteps > 1) or per job (domL > 0)
+    int domL = 0;                        // > 0: tree jobs of domL row tiles (see update_kernel)
     int64_t vcol = 0, tcol = 0, ecol = 0;
     unsigned* prog = nullptr;
 };
