@@ -180,6 +180,11 @@ tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const in
  * (capacity cap) and the length to *len. */
 tqr_status tqr_generate_guide(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len);
 
+/* Row split (tqr_options.row_split): owner g of ndev holds rows [r0[g], r0[g] + rows[g]) of an
+ * m-row single-column-tile matrix -- the contiguous tile rows [g p / ndev, (g+1) p / ndev),
+ * p = ceil(m / nb).  Host-only (used by tqr_create_ex and the multi-process CPU tests). */
+tqr_status tqr_row_split_ranges(int64_t m, int32_t nb, int32_t ndev, int64_t* r0, int64_t* rows);
+
 /* Measured average time (seconds) of one tile operation on a device (the paper's time_i(op),
  * P:L878-881): T = triangulation (GEQRT), E = elimination (TSQRT), UT = update for
  * triangulation (UNMQR), UE = update for elimination (TSMQR). */

@@ -73,6 +73,7 @@ def lib():
         L.tqr_schedule.argtypes = [i64, i64, i32, i32, P(i32), i32, i32, P(i32), i64, P(i64)]
         L.tqr_generate_guide.argtypes = [P(i32), i32, P(i32), i32, P(i32)]
         L.tqr_select_main.argtypes = [i32, P(TileTimes), P(i32)]
+        L.tqr_row_split_ranges.argtypes = [i64, i32, i32, P(i64), P(i64)]
         L.tqr_select_ndev.argtypes = [i32, i32, i32, i32, i32, P(TileTimes), P(ctypes.c_double), i32, P(i32),
                                       P(ctypes.c_double), P(i32)]
         L.tqr_kernel_stats.argtypes = [vp, i32, P(i64), P(ctypes.c_double), P(ctypes.c_double), i32]
@@ -80,7 +81,7 @@ def lib():
         L.tqr_launch_count.restype = i64
         for f in ("tqr_create", "tqr_create_ex", "tqr_factor", "tqr_load", "tqr_factor_tiles", "tqr_store_r",
                   "tqr_apply_qt", "tqr_solve_ls", "tqr_destroy", "tqr_nccl_unique_id", "tqr_schedule",
-                  "tqr_generate_guide", "tqr_kernel_stats", "tqr_select_main", "tqr_select_ndev"):
+                  "tqr_generate_guide", "tqr_kernel_stats", "tqr_select_main", "tqr_select_ndev", "tqr_row_split_ranges"):
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -89,7 +90,7 @@ def lib():
 EXPORTED = ["tqr_create", "tqr_create_ex", "tqr_factor", "tqr_load", "tqr_factor_tiles", "tqr_store_r",
             "tqr_apply_qt", "tqr_solve_ls", "tqr_destroy", "tqr_status_string", "tqr_last_error",
             "tqr_nccl_unique_id", "tqr_owner", "tqr_schedule", "tqr_generate_guide", "tqr_kernel_stats",
-            "tqr_launch_count", "tqr_select_main", "tqr_select_ndev"]
+            "tqr_launch_count", "tqr_select_main", "tqr_select_ndev", "tqr_row_split_ranges"]
 
 
 def _check(st: int, h=None):
@@ -217,6 +218,14 @@ def _times(times):
     for i, t in enumerate(times):
         arr[i] = TileTimes(*[float(x) for x in t])
     return arr
+
+
+def tqr_row_split_ranges(m, nb, ndev):
+    """Row blocks of a row-split plan: [(r0, rows)] per owner."""
+    r0 = (ctypes.c_int64 * ndev)()
+    rows = (ctypes.c_int64 * ndev)()
+    _check(lib().tqr_row_split_ranges(m, nb, ndev, r0, rows), None)
+    return list(zip(r0, rows))
 
 
 def tqr_select_main(times):

@@ -432,6 +432,17 @@ tqr_status tqr_destroy(tqr_plan h) {
     return TQR_OK;
 }
 
+tqr_status tqr_row_split_ranges(int64_t m, int32_t nb, int32_t ndev, int64_t* r0, int64_t* rows) {
+    if (m < 1 || nb < 1 || ndev < 1 || !r0 || !rows) return TQR_ERR_ARG;
+    const int64_t p = (m + nb - 1) / nb;
+    for (int g = 0; g < ndev; ++g) {
+        const int64_t t0 = g * p / ndev, t1 = (g + 1) * p / ndev;
+        r0[g] = std::min<int64_t>(t0 * nb, m);
+        rows[g] = std::min<int64_t>(t1 * nb, m) - r0[g];
+    }
+    return TQR_OK;
+}
+
 // Row-split plan (see tqr_options.row_split): owner g holds tile rows [g p / G, (g+1) p / G).
 static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
                                    const tqr_options& o, bool use_nccl, int world, tqr_plan* out) {
@@ -448,12 +459,11 @@ static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib,
     h->nccl_mode = use_nccl;
     h->profile = o.profile != 0;
     auto bail = [&](tqr_status st) { std::string e = h->err; tqr_destroy(h); g_create_error = e; return st; };
-    for (int g = 0; g < ndev; ++g) {
-        const int64_t t0 = g * p / ndev, t1 = (g + 1) * p / ndev;
-        h->rs_r0.push_back(t0 * nb);
-        h->rs_rows.push_back(std::min<int64_t>(t1 * nb, m) - t0 * nb);
-        if (h->rs_rows.back() < n) return bail(fail(h, TQR_ERR_UNSUPPORTED, "row split: owner %d gets %lld < n rows", g, (long long)h->rs_rows.back()));
-    }
+    h->rs_r0.resize(ndev);
+    h->rs_rows.resize(ndev);
+    tqr_row_split_ranges(m, nb, ndev, h->rs_r0.data(), h->rs_rows.data());
+    for (int g = 0; g < ndev; ++g)
+        if (h->rs_rows[g] < n) return bail(fail(h, TQR_ERR_UNSUPPORTED, "row split: owner %d gets %lld < n rows", g, (long long)h->rs_rows[g]));
     int cur = 0;
     cudaGetDevice(&cur);
     tqr_options co{};

@@ -111,3 +111,61 @@ def test_distributed_schedule_and_broadcast(tmp_path, world, guide):
     assert colnorm_rel_err(R, ref) <= 1e-10
     p = m // nb
     assert list(np.load(tmp_path / "bytes.npy")) == [8 * ((m - k * nb) * nb + (p - k) * ib * nb) for k in range(n // nb)]
+
+
+def _rowsplit_worker(rank, world, m, n, nb, ib, seed, port, out_dir):
+    """Row split (tqr_options.row_split) protocol with LAPACK tile kernels standing in for the
+    CUDA ones: rank g takes its rows from tqr_row_split_ranges, factors them as a flat TS chain
+    (dgeqrt + dtpqrt), the owners' nb x n triangular factors are all-gathered (the NCCL
+    all-gather of the library), and rank 0 factors the stacked triu(R_g)."""
+    import sys
+    sys.path.insert(0, ROOT)
+    import scipy.linalg.lapack as lap
+    import synthetic
+    import paper_conf_icpp_kimp13_b200 as tqr
+
+    dist.init_process_group("gloo", init_method="tcp://127.0.0.1:%d" % port, rank=rank, world_size=world)
+    A = synthetic.gaussian(m, n, seed)
+    ranges = tqr.tqr_row_split_ranges(m, nb, world)
+    r0, rows = ranges[rank]
+    blk = np.zeros((-(-rows // nb) * nb, n))
+    blk[:rows] = A[r0:r0 + rows]
+    a, t, info = lap.dgeqrt(ib, np.asfortranarray(blk[:nb]))
+    assert info == 0
+    top = np.triu(a)
+    for i in range(1, blk.shape[0] // nb):
+        r, b, t, info = lap.dtpqrt(0, ib, top, np.asfortranarray(blk[i * nb:(i + 1) * nb]))
+        assert info == 0
+        top = np.triu(r)
+    send = torch.from_numpy(np.ascontiguousarray(top[:nb, :n]))
+    recv = [torch.zeros_like(send) for _ in range(world)]
+    dist.all_gather(recv, send)
+    if rank == 0:
+        stk = np.vstack([x.numpy() for x in recv])             # ndev*nb x n, triu blocks
+        a, t, info = lap.dgeqrt(ib, np.asfortranarray(stk[:nb]))
+        top = np.triu(a)
+        for g in range(1, world):
+            r, b, t, info = lap.dtpqrt(0, ib, top, np.asfortranarray(stk[g * nb:(g + 1) * nb]))
+            top = np.triu(r)
+        np.save(os.path.join(out_dir, "R.npy"), top[:n, :n])
+        np.save(os.path.join(out_dir, "ranges.npy"), np.array(ranges))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,m", [(2, 1024), (3, 1000)])
+def test_row_split_protocol(tmp_path, world, m):
+    import oracle
+    import synthetic
+    from conftest import colnorm_rel_err
+    from paper_conf_icpp_kimp13_b200 import build
+    build.build()
+    n, nb, ib, seed = 64, 64, 16, 4343
+    mp.spawn(_rowsplit_worker, args=(world, m, n, nb, ib, seed, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    R = np.load(tmp_path / "R.npy")
+    ref = oracle.qr(synthetic.gaussian(m, n, seed)).R
+    assert colnorm_rel_err(R, ref) <= 1e-10
+    ranges = np.load(tmp_path / "ranges.npy")
+    assert ranges[0][0] == 0 and sum(r for _, r in ranges) == m                 # contiguous cover
+    assert all(ranges[g][0] + ranges[g][1] == ranges[g + 1][0] for g in range(world - 1))
+    assert all(r0 % nb == 0 and r >= n for r0, r in ranges)
