@@ -1,7 +1,9 @@
 """compute-sanitizer racecheck / synccheck / memcheck over small factorizations (SURVEY sec. 5:
 race detection).  Covers the inter-CTA flag wavefront of the panel kernel, the cp.async.bulk /
-mbarrier staging and the shared-memory reductions of both kernels, apply_qt and the logical-
-device (peer-copy broadcast) path."""
+mbarrier staging and the shared-memory reductions of both kernels, apply_qt (wavefront) and the
+logical-device (peer-copy broadcast) path, the lookahead beside its panel, the tile back
+substitution, streamed host I/O, tree jobs with the two-level merge, the streamed tall factor and
+the row split."""
 import os
 import shutil
 import subprocess
@@ -25,5 +27,5 @@ def test_sanitizer_clean(tool):
                          cwd=ROOT, capture_output=True, text=True, timeout=900)
     text = out.stdout + out.stderr
     assert out.returncode == 0, text[-3000:]
-    assert "ok 1024 1024 512 32" in text, text[-3000:]
+    assert "ok 1024 1024 512 32" in text and "ok extra" in text, text[-3000:]
     assert ("0 errors" in text) or ("0 hazards displayed (0 errors" in text), text[-3000:]

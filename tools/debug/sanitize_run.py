@@ -14,3 +14,27 @@ for (m, n, nb, ib) in [(256, 256, 64, 16), (512, 256, 128, 32), (1024, 1024, 512
         Ad = torch.from_numpy(np.ascontiguousarray(A.T)).cuda().t()
         p.factor(Ad)
     print("ok", m, n, nb, ib, flush=True)
+# round-1 additions: tile back substitution, streamed host I/O, tree jobs + two-level merge,
+# streamed tall factor, row split
+m, n, nb, ib = 512, 256, 128, 32
+A = synthetic.gaussian(m, n, 5)
+with tqr.Plan(m, n, nb, ib) as p:
+    Ah = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    p.factor(Ah)
+    B = torch.from_numpy(np.ascontiguousarray(synthetic.gaussian(m, 40, 6).T)).cuda().t()
+    p.solve_ls(B)
+A = synthetic.gaussian(2048, 128, 7)
+with tqr.Plan(2048, 128, 64, 16, tree_domain=1, tree_group=4) as p:
+    Ad = torch.from_numpy(np.ascontiguousarray(A.T)).cuda().t()
+    p.factor(Ad)
+    B = torch.from_numpy(np.ascontiguousarray(synthetic.gaussian(2048, 3, 8).T)).cuda().t()
+    p.apply_qt(B, "T"); p.apply_qt(B, "N")
+os.environ["TQR_TREE_ONE_CTA"] = "1"
+A = synthetic.gaussian(2048, 64, 9)
+with tqr.Plan(2048, 64, 64, 16) as p:
+    Ah = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    p.factor(Ah)
+with tqr.Plan(2048, 64, 64, 16, ndev=2, logical_devices=True, row_split=1) as p:
+    Ad = torch.from_numpy(np.ascontiguousarray(A.T)).cuda().t()
+    p.factor(Ad)
+print("ok extra", flush=True)
