@@ -382,6 +382,10 @@ def main():
                         "traffic": prof.get("dram_bytes_per_launch"), "traffic_note": prof.get("note"),
                         "peak_source": peak_src, "launches_per_step": pcount // K,
                         "busy_ms_per_step": round(pms / K, 3), "share_of_step": round(pms / K / ms, 3)}
+            if pach / peak < 0.1:
+                roofline["note"] = ("the panel chain (GEQRT + TSQRT wavefront, one ib block after another) is "
+                                    "latency-bound here (SURVEY 8(d): no roofline claim for C1/C2): the step is "
+                                    "the critical path of the flat TS panels, not a throughput limit")
         line = {
             "metric": METRIC,
             "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
