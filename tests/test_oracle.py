@@ -117,6 +117,34 @@ def test_lapack_agreement(m, n):
     assert colnorm_rel_err(f.R, R_lapack) < 1e-13
 
 
+@pytest.mark.parametrize("scale", [1e300, 1e200, 1e-200, 1e-300])
+def test_extreme_scaling_matches_lapack(scale):
+    """Reading Q26: ||a_k|| (Alg. 1 lines 6 and 8) is the Euclidean norm, computed without
+    overflow or underflow.  sqrt(sum x^2) is inf for entries ~1e200 and 0 for ~1e-200 (tau = 0,
+    nothing eliminated); LAPACK's dlarfg/dnrm2 scale.  R(cA) = c R(A) for a power-of-ten c, so
+    the oracle's R of the scaled matrix must match LAPACK's and c x the unscaled oracle R."""
+    A = synthetic.gaussian(96, 64, 22)
+    As = A * scale
+    f = oracle.qr(As)
+    assert np.all(np.isfinite(f.R))
+    R_lapack = np.linalg.qr(As, mode="r")
+    assert colnorm_rel_err(f.R, R_lapack) < 1e-13
+    assert colnorm_rel_err(f.R / scale, oracle.qr(A).R) < 1e-13
+    Q = f.thin_q()
+    assert np.linalg.norm(Q.T @ Q - np.eye(64)) < 1e-13
+
+
+def test_scaled_norm_bitwise_in_normal_range():
+    """Power-of-two scaling is exact: in the normal range the scaled norm is bitwise the plain
+    sqrt(sum x^2) of Alg. 1 (the closed forms above pin the same arithmetic)."""
+    A = synthetic.gaussian(50, 1, 23) * 3.0
+    f = oracle.qr(A)
+    s = 0.0
+    for x in A[:, 0]:                        # ascending rows, as Alg. 1's sum is taken
+        s += float(x) * float(x)
+    assert abs(f.R[0, 0]) == np.sqrt(s)
+
+
 def test_thin_q_orthogonal_and_reconstructs():
     A = synthetic.gaussian(300, 120, 13)
     f = oracle.qr(A)
