@@ -10,10 +10,13 @@ step   : one pass of the whole hot path over the config
          updates, lookahead, broadcasts) + tqr_store_r (R out).  Input resident in HBM.
 e2e    : the same through tqr_factor on a PINNED HOST A (H2D of A and D2H of R inside the
          timed region, pipelined with the factorization by the library).
-N > 1  : launched by torchrun; one process per GPU, column tiles partitioned by a guide array
-         (Eq. 12; --guide: cyclic {0..N-1}, or pairs {0,0,1,1,..} -- default for N >= 8), panels
-         broadcast with NCCL; a single column tile (C4) is split by rows instead (row split).
-         Strong scaling (same matrix).
+N > 1  : one process per GPU (bench.py starts the N ranks itself with torchrun when WORLD_SIZE is
+         unset), column tiles partitioned by a guide array (Eq. 12; --guide: cyclic {0..N-1}, or
+         pairs {0,0,1,1,..} -- default for N >= 8); each panel travels from its owner to the other
+         ranks by the library's CUDA-IPC transport (device-to-device copies into the receivers'
+         IPC-mapped slots over NVLink, ordered by stream flags; --transport nccl: ncclBroadcast);
+         a single column tile (C4) is split by rows instead (row split).  Strong scaling (same
+         matrix).  More ranks than GPUs (testing on one GPU): ranks share GPUs, n_gpus counts GPUs.
 --impl reference : the CPU oracle (Algorithm 1, oracle/) timed on this host's cores on a
          bounded sample of the same workload (first 2048 columns of the config's matrix).
 """
@@ -206,21 +209,42 @@ def main():
                     help="also time tqr_solve_ls with this many right-hand sides (NEXT-3; 'solve' key)")
     ap.add_argument("--tree-group", type=int, default=0,
                     help="tree merge: 0 auto (two-level for >= 16 domains), -1 flat chain, G > 1 groups of G")
+    ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
+                    help="N > 1 panel transport: ipc = the library's own CUDA-IPC peer copies + stream "
+                         "flags (default); nccl = ncclBroadcast")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
 
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world == 1 and args.gpus > 1:
+        # started without torchrun: launch the N ranks ourselves (one process per GPU), rank 0
+        # prints the JSON line
+        import socket
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes", "1", "--nproc-per-node", str(args.gpus),
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd)
+
     import torch
     import paper_conf_icpp_kimp13_b200 as tqr
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local_rank)
+    ndevices = torch.cuda.device_count()
+    device = local_rank % ndevices          # more ranks than GPUs: ranks share GPUs (tests / smoke)
+    torch.cuda.set_device(device)
+    shared = world > ndevices
+    n_gpus = min(world, ndevices)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if shared or args.transport == "ipc":
+            dist.init_process_group("gloo")          # host-side handshake + barriers only
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", device))
 
     m, n, nb, ib, seed = CONFIGS[args.config]
     f32 = args.dtype == "f32"
@@ -235,7 +259,7 @@ def main():
     Rout = torch.empty((n, m), dtype=tdt, device="cuda").t()
 
     nccl_id = None
-    if world > 1:
+    if world > 1 and args.transport == "nccl":
         obj = [tqr.tqr_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
@@ -243,8 +267,12 @@ def main():
     guide = [d for d in range(world) for _ in range(2 if gmode == "pairs" else 1)]
     plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, guide=guide,
                     rank=rank, world=world, nccl_id=nccl_id,
+                    transport=("nccl" if args.transport == "nccl" else "ipc") if world > 1 else "auto",
                     lookahead=not args.no_lookahead, profile=True, tree_domain=args.tree,
                     tree_group=args.tree_group)
+    if world > 1 and args.transport == "ipc":
+        plan.connect()
+    pflags = plan.flags()
 
     def step(Ain, Aout):
         plan.load(Ain)
@@ -258,7 +286,9 @@ def main():
     def max_over_ranks(x):
         if dist is None:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64)
+        if dist.get_backend() == "nccl":
+            t = t.cuda()
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
@@ -271,7 +301,7 @@ def main():
 
     stream = torch.cuda.current_stream()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local_rank) as clk:
+    with ClockSampler(device) as clk:
         barrier()
         torch.cuda.synchronize()
         ev0.record(stream)
@@ -323,7 +353,7 @@ def main():
     # ---- least squares throughput (NEXT-3): Q^T B (update kernel) + tile back substitution on a
     # device-resident B of --solve columns; B restored from a pristine copy between calls (untimed)
     solve = None
-    if args.solve > 0 and world == 1:
+    if args.solve > 0:
         nr = args.solve
         gen_b = torch.Generator(device="cuda").manual_seed(seed + 1)
         B0 = torch.randn((nr, m), dtype=tdt, device="cuda", generator=gen_b).t()
@@ -388,15 +418,19 @@ def main():
                                     "the critical path of the flat TS panels, not a throughput limit")
         line = {
             "metric": METRIC,
-            "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": W,
+            "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": n_gpus, "steps": K, "warmup": W,
             "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
-            ("pct_fp32_ffma_peak" if f32 else "pct_fp64_peak"): round(100.0 * value / 1e3 / (peak * world), 2),
+            ("pct_fp32_ffma_peak" if f32 else "pct_fp64_peak"): round(100.0 * value / 1e3 / (peak * n_gpus), 2),
             "config": {"workload": args.config, "m": m, "n": n, "nb": nb, "ib": ib, "seed": seed,
                        "input": "torch.randn N(0,1) %s on device (seeded)" % args.dtype, "guide": guide,
-                       "parallelism": ("row-split x%d (per-rank TS trees + NCCL all-gather of the R factors, "
-                                       "stage-2 merge on rank 0)" % world) if (n <= nb and world > 1) else
-                                      "col-cyclic x%d" % world, "lookahead": not args.no_lookahead,
+                       "parallelism": ("row-split x%d (per-rank TS trees + %s gather of the R factors, "
+                                       "stage-2 merge on rank 0)" % (world, "IPC" if pflags & tqr.PLAN_IPC else "NCCL"))
+                                      if pflags & tqr.PLAN_ROW_SPLIT else
+                                      ("col-%s x%d%s" % (gmode, world, (", %s panel transport" %
+                                                                        ("CUDA-IPC" if pflags & tqr.PLAN_IPC else "NCCL"))
+                                                         if world > 1 else "")),
+                       "ranks": world, "ranks_share_gpus": shared, "lookahead": not args.no_lookahead,
                        "tree": args.tree, "tree_group": args.tree_group,
                        "l2": "inputs larger than L2 (%.1f GiB >> 126 MB)" % (es * m * n / 2 ** 30)
                        if es * m * n > L2_BYTES else "input fits L2 (no flush)"},

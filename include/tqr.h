@@ -54,10 +54,11 @@ typedef struct {
      * guide-array partition and broadcast ordering on one GPU.  0: owner d uses CUDA
      * device d (single-process) or this process's device (multi-process). */
     int32_t logical_devices;
-    /* Multi-process (NCCL) mode, one process per GPU: world > 1 (or world <= 1 with a non-NULL
-     * nccl_id: a single-rank communicator), this process is `rank`; ndev must equal
-     * max(world, 1).  nccl_id points to the 128-byte ncclUniqueId produced by
-     * tqr_nccl_unique_id() on rank 0 and shared out of band (e.g. torch.distributed). */
+    /* Multi-process mode, one process per owner: world > 1 (or world <= 1 with a non-NULL
+     * nccl_id: a single-rank NCCL communicator), this process is `rank`; ndev must equal
+     * max(world, 1).  The panel transport is chosen by `transport` (below): NCCL needs nccl_id,
+     * the 128-byte ncclUniqueId produced by tqr_nccl_unique_id() on rank 0 and shared out of band
+     * (e.g. torch.distributed); IPC needs the tqr_ipc_handle / tqr_ipc_connect exchange. */
     int32_t rank;
     int32_t world;
     const void* nccl_id;
@@ -86,7 +87,20 @@ typedef struct {
      * owner), 1 = force, -1 = off (column partition: owner(0) does all the work).  Row-split
      * plans support tqr_factor / tqr_load / tqr_factor_tiles / tqr_store_r only. */
     int32_t row_split;
+    /* Multi-process panel transport.  TQR_TRANSPORT_AUTO (0): NCCL when nccl_id is
+     * given, otherwise IPC.  TQR_TRANSPORT_NCCL (1): ncclBroadcast of every panel from its owner
+     * on a comm stream (one GPU per rank).  TQR_TRANSPORT_IPC (2): the panel owner copies V/T
+     * straight into each receiving rank's CUDA-IPC-mapped receive slot (NVLink peer memory, or the
+     * same HBM when several ranks share one GPU) and orders the copy with stream-ordered 64-bit
+     * flags (cuStreamWaitValue64 / cuStreamWriteValue64): no NCCL, no SM spent on the transfer,
+     * any number of ranks per GPU.  An IPC plan must be connected (tqr_ipc_handle on every rank,
+     * all blobs exchanged out of band, tqr_ipc_connect) before its first factor. */
+    int32_t transport;
 } tqr_options;
+
+#define TQR_TRANSPORT_AUTO 0
+#define TQR_TRANSPORT_NCCL 1
+#define TQR_TRANSPORT_IPC 2
 
 /*
  * Create a plan for the QR factorisation of an m x n matrix.
@@ -97,7 +111,8 @@ typedef struct {
  *   nb        : tile size (square tiles); supported 64, 128, 256, 512.
  *   ib        : inner blocking of the compact-WY T factors; 1 <= ib <= nb, nb % ib == 0;
  *               supported 16, 32.
- *   dtype     : TQR_F64 (TQR_F32 returns TQR_ERR_UNSUPPORTED in this build).
+ *   dtype     : TQR_F64 or TQR_F32 (FP32 tiles and updates; each panel is factored in FP64 and
+ *               rounded once, reading Q9).  Tree mode (tree_domain > 0) is FP64 only.
  *   ndev      : number of column-tile owners (devices).
  *   guide     : distribution guide array (Alg. 4), entries in [0, ndev); column tile j is
  *               owned by guide[j % guide_len] (Eq. 12).  NULL -> {0, 1, ..., ndev-1}.
@@ -137,7 +152,14 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda);
  * B (m x nrhs, ldb >= m) <- Q^T B (trans 'T') or Q B (trans 'N'), with Q from the last
  * tqr_factor (Alg. 1 lines 13-14 read for the tiled factorisation).  Rows 0..n-1 of Q^T B
  * (and Q [C; 0]) are unique; rows n..m-1 of Q^T B depend on the tile algorithm.
- * TQR_ERR_STATE before a successful factor.  Multi-process plans: TQR_ERR_UNSUPPORTED.
+ * TQR_ERR_STATE before a successful factor.
+ * Several owners (logical devices, several GPUs, or ranks): the first apply/solve after a factor
+ * gathers every panel's reflectors, T factors and R tiles onto the caller's device (peer copies;
+ * ncclBroadcast from each column's owner; or IPC pulls from the owners' memory), then applies
+ * there.  Multi-process plans: a collective -- every rank calls it with its own full B and gets
+ * the full result; an IPC plan returns only when every rank has finished its pulls, so the next
+ * factor cannot overwrite reflectors a peer is still reading.  Row-split plans: the owners apply
+ * their blocks' Q_g, then the stage-2 plan's Q to the stacked top rows (single process only).
  */
 tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs);
 
@@ -161,6 +183,34 @@ const char* tqr_last_error(tqr_plan h);
 /* Write a fresh 128-byte ncclUniqueId into id[0..127] (rank 0 of a multi-process plan).
  * TQR_ERR_NCCL if libnccl.so.2 cannot be loaded. */
 tqr_status tqr_nccl_unique_id(void* id128);
+
+/* CUDA-IPC transport handshake (tqr_options.transport = TQR_TRANSPORT_IPC, multi-process).
+ * tqr_ipc_handle writes this rank's export blob (IPC handles of its receive slots, flag block and
+ * reflector storage) into buf (capacity cap bytes; buf NULL = size query) and its size to *len
+ * (the same on every rank).  The application all-gathers the blobs in rank order (e.g.
+ * torch.distributed.all_gather_object) and passes the world * len concatenation to
+ * tqr_ipc_connect, which opens every peer's memory (cudaIpcMemLazyEnablePeerAccess) and arms
+ * the transfer flags.  TQR_ERR_STATE on a non-IPC plan or a second connect; TQR_ERR_ARG on a
+ * blob of the wrong size or rank order; TQR_ERR_CUDA if a handle cannot be opened. */
+tqr_status tqr_ipc_handle(tqr_plan h, void* buf, int64_t cap, int64_t* len);
+tqr_status tqr_ipc_connect(tqr_plan h, const void* all, int64_t len);
+
+/* The operations the last tqr_factor_tiles issued on this rank, in issue order, as the same
+ * 5-int32 records tqr_schedule produces ({op, k, i, j, root}; UPDATE records one per column, in
+ * the order the columns' launches were enqueued).  The executor consumes tqr_schedule's list,
+ * so per step k the records are the schedule's (tests compare them).  cap/count as tqr_schedule. */
+tqr_status tqr_issued_ops(tqr_plan h, int32_t* ops, int64_t cap, int64_t* count);
+
+/* How the plan executes, as a bit mask (0 for NULL): TQR_PLAN_ROW_SPLIT (single column tile split by
+ * rows across the owners), TQR_PLAN_TREE (TS domains + TT merges), TQR_PLAN_MULTIPROC (one process
+ * per owner), TQR_PLAN_IPC / TQR_PLAN_NCCL (its panel transport), TQR_PLAN_F32. */
+#define TQR_PLAN_ROW_SPLIT 1
+#define TQR_PLAN_TREE 2
+#define TQR_PLAN_MULTIPROC 4
+#define TQR_PLAN_IPC 8
+#define TQR_PLAN_NCCL 16
+#define TQR_PLAN_F32 32
+int32_t tqr_plan_flags(tqr_plan h);
 
 /* Owner of column tile j under the plan's guide array (Eq. 12), or -1 if j is out of range. */
 int32_t tqr_owner(tqr_plan h, int64_t j);
@@ -211,9 +261,12 @@ tqr_status tqr_select_ndev(int32_t M, int32_t N, int32_t T, int32_t elem_size, i
                            double* Tp, int32_t* pbest);
 
 /* Device-time statistics of the plan's kernels since the last reset (opt.profile = 1):
- * which = 0 update (UNMQR+TSMQR) kernel, 1 panel (GEQRT+TSQRT) kernel, 2 layout kernels,
- * 3 broadcast.  *count launches, *ms summed CUDA-event milliseconds, *flops algorithmic
- * flops of those launches.  reset != 0 clears after reading. */
+ * which = 0 update (UNMQR+TSMQR) kernel, 1 panel (GEQRT+TSQRT) kernel, 2 layout kernels (a1
+ * to_tiles in tqr_load, a8 from_tiles in tqr_store_r), 3 panel transfers (BCAST: NCCL
+ * broadcast, IPC copies or peer copies, from the transfer's start to the receive completing).
+ * *count launches (transfers), *ms device-busy CUDA-event milliseconds (union of the intervals:
+ * overlapping launches are not double counted), *flops algorithmic flops (which = 0, 1) or
+ * bytes moved (which = 2, 3).  reset != 0 clears after reading. */
 tqr_status tqr_kernel_stats(tqr_plan h, int32_t which, int64_t* count, double* ms, double* flops, int32_t reset);
 
 /* Number of kernel launches the plan issued since the last call (then resets). */

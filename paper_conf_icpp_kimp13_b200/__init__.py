@@ -17,12 +17,13 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libtqr.so")
+LIB_PATH = os.environ.get("TQR_LIB") or os.path.join(_PKG, "libtqr.so")   # TQR_LIB: probe builds only
 
 TQR_F64, TQR_F32 = 0, 1
 STATUS = {0: "TQR_OK", 1: "TQR_ERR_ARG", 2: "TQR_ERR_ALLOC", 3: "TQR_ERR_CUDA", 4: "TQR_ERR_NCCL",
           5: "TQR_ERR_STATE", 6: "TQR_ERR_SINGULAR", 7: "TQR_ERR_UNSUPPORTED"}
 OP_PANEL, OP_BCAST, OP_UPDATE = 0, 1, 2
+TRANSPORT = {"auto": 0, "nccl": 1, "ipc": 2}
 
 
 class TqrError(RuntimeError):
@@ -35,7 +36,7 @@ class Options(ctypes.Structure):
     _fields_ = [("logical_devices", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("nccl_id", ctypes.c_void_p), ("no_lookahead", ctypes.c_int32), ("profile", ctypes.c_int32),
                 ("tree_domain", ctypes.c_int32), ("tree_group", ctypes.c_int32),
-                ("row_split", ctypes.c_int32)]
+                ("row_split", ctypes.c_int32), ("transport", ctypes.c_int32)]
 
 
 class TileTimes(ctypes.Structure):
@@ -79,9 +80,15 @@ def lib():
         L.tqr_kernel_stats.argtypes = [vp, i32, P(i64), P(ctypes.c_double), P(ctypes.c_double), i32]
         L.tqr_launch_count.argtypes = [vp]
         L.tqr_launch_count.restype = i64
+        L.tqr_ipc_handle.argtypes = [vp, vp, i64, P(i64)]
+        L.tqr_ipc_connect.argtypes = [vp, vp, i64]
+        L.tqr_issued_ops.argtypes = [vp, P(i32), i64, P(i64)]
+        L.tqr_plan_flags.argtypes = [vp]
+        L.tqr_plan_flags.restype = i32
         for f in ("tqr_create", "tqr_create_ex", "tqr_factor", "tqr_load", "tqr_factor_tiles", "tqr_store_r",
                   "tqr_apply_qt", "tqr_solve_ls", "tqr_destroy", "tqr_nccl_unique_id", "tqr_schedule",
-                  "tqr_generate_guide", "tqr_kernel_stats", "tqr_select_main", "tqr_select_ndev", "tqr_row_split_ranges"):
+                  "tqr_generate_guide", "tqr_kernel_stats", "tqr_select_main", "tqr_select_ndev", "tqr_row_split_ranges",
+                  "tqr_ipc_handle", "tqr_ipc_connect", "tqr_issued_ops"):
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -90,7 +97,9 @@ def lib():
 EXPORTED = ["tqr_create", "tqr_create_ex", "tqr_factor", "tqr_load", "tqr_factor_tiles", "tqr_store_r",
             "tqr_apply_qt", "tqr_solve_ls", "tqr_destroy", "tqr_status_string", "tqr_last_error",
             "tqr_nccl_unique_id", "tqr_owner", "tqr_schedule", "tqr_generate_guide", "tqr_kernel_stats",
-            "tqr_launch_count", "tqr_select_main", "tqr_select_ndev", "tqr_row_split_ranges"]
+            "tqr_launch_count", "tqr_select_main", "tqr_select_ndev", "tqr_row_split_ranges",
+            "tqr_ipc_handle", "tqr_ipc_connect", "tqr_issued_ops", "tqr_plan_flags"]
+PLAN_ROW_SPLIT, PLAN_TREE, PLAN_MULTIPROC, PLAN_IPC, PLAN_NCCL, PLAN_F32 = 1, 2, 4, 8, 16, 32
 
 
 def _check(st: int, h=None):
@@ -106,12 +115,26 @@ def _i32_array(vals):
 
 
 _PLAN_DTYPE = {}   # plan handle value -> TQR_F64 / TQR_F32 (argument checking only)
+_PLAN_SHAPE = {}   # plan handle value -> (m, n) (argument checking only)
 
 
-def _ptr_ld(x, rows: int, h=None):
+def _check_shape(x, need_rows, need_cols):
+    """The library reads / writes need_rows x need_cols elements through the pointer: refuse arrays
+    that are smaller (would be an out-of-bounds host or device access)."""
+    shp = tuple(x.shape)
+    rows = shp[0] if len(shp) >= 1 else 0
+    cols = shp[1] if len(shp) >= 2 else 1
+    if rows < need_rows or cols < need_cols:
+        raise ValueError("array of shape %s is smaller than the plan's %d x %d" % (shp, need_rows, need_cols))
+
+
+def _ptr_ld(x, rows: int, h=None, need_cols=None):
     """(pointer, leading dimension) of a column-major 2-D torch tensor or numpy array whose element
-    type matches the plan's dtype."""
+    type matches the plan's dtype (and, for a known plan, at least m rows and need_cols columns)."""
     want = _PLAN_DTYPE.get(getattr(h, "value", None), None)
+    shape = _PLAN_SHAPE.get(getattr(h, "value", None), None)
+    if shape is not None:
+        _check_shape(x, shape[0], shape[1] if need_cols is None else need_cols)
     try:
         import torch
         if isinstance(x, torch.Tensor):
@@ -141,10 +164,11 @@ def _ptr_ld(x, rows: int, h=None):
 
 # ------------------------------------------------------------------ ABI-named functions
 def tqr_create(m, n, nb, ib, dtype=TQR_F64, ndev=1, guide=None, logical_devices=False, rank=0, world=1,
-               nccl_id=None, lookahead=True, profile=False, tree_domain=0, tree_group=0, row_split=0):
+               nccl_id=None, lookahead=True, profile=False, tree_domain=0, tree_group=0, row_split=0,
+               transport="auto"):
     g, glen = _i32_array(guide)
     opt = Options(int(bool(logical_devices)), int(rank), int(world), None, int(not lookahead), int(bool(profile)),
-                  int(tree_domain), int(tree_group), int(row_split))
+                  int(tree_domain), int(tree_group), int(row_split), int(TRANSPORT[transport]))
     idbuf = None
     if nccl_id is not None:
         idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128)
@@ -154,6 +178,7 @@ def tqr_create(m, n, nb, ib, dtype=TQR_F64, ndev=1, guide=None, logical_devices=
                              ctypes.byref(h))
     _check(st, None)
     _PLAN_DTYPE[h.value] = int(dtype)
+    _PLAN_SHAPE[h.value] = (int(m), int(n))
     return h
 
 
@@ -177,20 +202,21 @@ def tqr_store_r(h, A):
 
 
 def tqr_apply_qt(h, B, trans="T"):
-    ptr, ld = _ptr_ld(B, B.shape[0], h)
     nrhs = 1 if len(B.shape) == 1 else B.shape[1]
+    ptr, ld = _ptr_ld(B, B.shape[0], h, need_cols=nrhs)
     _check(lib().tqr_apply_qt(h, trans.encode()[:1], ptr, ld, nrhs), h)
 
 
 def tqr_solve_ls(h, B):
-    ptr, ld = _ptr_ld(B, B.shape[0], h)
     nrhs = 1 if len(B.shape) == 1 else B.shape[1]
+    ptr, ld = _ptr_ld(B, B.shape[0], h, need_cols=nrhs)
     _check(lib().tqr_solve_ls(h, ptr, ld, nrhs), h)
 
 
 def tqr_destroy(h):
     if h:
         _PLAN_DTYPE.pop(h.value, None)
+        _PLAN_SHAPE.pop(h.value, None)
         lib().tqr_destroy(h)
 
 
@@ -198,6 +224,30 @@ def tqr_nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(lib().tqr_nccl_unique_id(buf), None)
     return buf.raw
+
+
+def tqr_ipc_handle(h) -> bytes:
+    """This rank's CUDA-IPC export blob (IPC transport, multi-process)."""
+    ln = ctypes.c_int64()
+    _check(lib().tqr_ipc_handle(h, None, 0, ctypes.byref(ln)), h)
+    buf = ctypes.create_string_buffer(ln.value)
+    _check(lib().tqr_ipc_handle(h, buf, ln.value, ctypes.byref(ln)), h)
+    return buf.raw
+
+
+def tqr_ipc_connect(h, blobs):
+    """Open every rank's export (blobs: list of bytes in rank order)."""
+    allb = b"".join(bytes(b) for b in blobs)
+    buf = ctypes.create_string_buffer(allb, len(allb))
+    _check(lib().tqr_ipc_connect(h, buf, len(allb)), h)
+
+
+def tqr_issued_ops(h):
+    cnt = ctypes.c_int64()
+    _check(lib().tqr_issued_ops(h, None, 0, ctypes.byref(cnt)), h)
+    buf = (ctypes.c_int32 * max(1, 5 * cnt.value))()
+    _check(lib().tqr_issued_ops(h, buf, cnt.value, ctypes.byref(cnt)), h)
+    return [tuple(buf[5 * i: 5 * i + 5]) for i in range(cnt.value)]
 
 
 def tqr_owner(h, j):
@@ -293,6 +343,27 @@ class Plan:
 
     def owner(self, j):
         return tqr_owner(self.h, j)
+
+    def ipc_handle(self):
+        return tqr_ipc_handle(self.h)
+
+    def ipc_connect(self, blobs):
+        tqr_ipc_connect(self.h, blobs)
+
+    def connect(self, group=None):
+        """IPC transport: exchange the export blobs over torch.distributed (all_gather_object on
+        `group`) and connect.  Host-side handshake only; no data moves."""
+        import torch.distributed as dist
+        blobs = [None] * dist.get_world_size(group)
+        dist.all_gather_object(blobs, self.ipc_handle(), group=group)
+        self.ipc_connect(blobs)
+
+    def issued_ops(self):
+        return tqr_issued_ops(self.h)
+
+    def flags(self):
+        """TQR_PLAN_* bit mask (row split, tree, multi-process, transport, FP32)."""
+        return int(lib().tqr_plan_flags(self.h))
 
     def kernel_stats(self, which, reset=False):
         return tqr_kernel_stats(self.h, which, reset)

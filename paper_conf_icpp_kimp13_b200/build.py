@@ -26,6 +26,7 @@ SOURCES = [
     os.path.join(CSRC, "kernels", "qr_kernels.cu"),
     os.path.join(CSRC, "kernels", "qr_kernels_f32.cu"),
     os.path.join(CSRC, "kernels", "trsm.cu"),
+    os.path.join(CSRC, "tqr_signal.cu"),
     os.path.join(CSRC, "tqr_api.cpp"),
     os.path.join(CSRC, "tqr_model.cpp"),
 ]

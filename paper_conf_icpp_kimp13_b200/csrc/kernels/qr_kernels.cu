@@ -129,14 +129,22 @@ __global__ void __launch_bounds__(kThreads, 1) panel_kernel(PanelArgs a) {
         Slice<NB, IB, IB> Xf;
         Xf.load_cg(Ai + (int64_t)b * IB * NB, NB);
         if (ge) {
-            factor_block<NB, IB, true>(Xf, sf, b * IB);
+            // rare redo with scaled norms (reading Q26) from the block as loaded (nobody else writes
+            // its rows >= b*IB; rows above are R, untouched by a GEQRT block)
+            if (factor_block<NB, IB, true>(Xf, sf, b * IB)) {
+                Xf.load_cg(Ai + (int64_t)b * IB * NB, NB);
+                factor_block<NB, IB, true, true>(Xf, sf, b * IB);
+            }
         } else {
             for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
                 const int c = idx / IB, j = idx % IB;
                 sf.Rsm[c * IB + j] = (j >= c) ? ld_cg(Akk + (int64_t)(b * IB + j) * NB + b * IB + c) : 0.0;
             }
             __syncthreads();
-            factor_block<NB, IB, false>(Xf, sf, b * IB);
+            if (factor_block<NB, IB, false>(Xf, sf, b * IB)) {
+                Xf.load_cg(Ai + (int64_t)b * IB * NB, NB);
+                factor_block<NB, IB, false, true>(Xf, sf, b * IB);
+            }
         }
         TQR_PP(2);
         // publish: reflectors (LAPACK layout in the tile), their stage image (TSQRT: V2 of tile i;
@@ -227,15 +235,40 @@ __global__ void __launch_bounds__(kThreads, 1) domain_kernel(DomainArgs a) {
             }
             __syncthreads();   // top rows written by the applies -> Rsm reads below
             TQR_PP(4);
+            // X (after the applies) is kept in the idle staging area for the rare scaled redo (Q26)
+            double* keep = &sf.Vst[0][0][0][0];
+            static_assert(sizeof(sf.Vst) / sizeof(double) >= NB * IB, "redo copy of the block");
+#pragma unroll
+            for (int mf = 0; mf < IB / 8; ++mf)
+#pragma unroll
+                for (int nf = 0; nf < G::NF; ++nf) {
+                    keep[((mf * G::NF + nf) * 2 + 0) * kThreads + threadIdx.x] = X.acc[mf][nf][0];
+                    keep[((mf * G::NF + nf) * 2 + 1) * kThreads + threadIdx.x] = X.acc[mf][nf][1];
+                }
+            auto restore = [&]() {
+#pragma unroll
+                for (int mf = 0; mf < IB / 8; ++mf)
+#pragma unroll
+                    for (int nf = 0; nf < G::NF; ++nf) {
+                        X.acc[mf][nf][0] = keep[((mf * G::NF + nf) * 2 + 0) * kThreads + threadIdx.x];
+                        X.acc[mf][nf][1] = keep[((mf * G::NF + nf) * 2 + 1) * kThreads + threadIdx.x];
+                    }
+            };
             if (ge) {
-                factor_block<NB, IB, true>(X, sf, b * IB);
+                if (factor_block<NB, IB, true>(X, sf, b * IB)) {
+                    restore();
+                    factor_block<NB, IB, true, true>(X, sf, b * IB);
+                }
             } else {
                 for (int idx = threadIdx.x; idx < IB * IB; idx += kThreads) {
                     const int c = idx / IB, j = idx % IB;
                     sf.Rsm[c * IB + j] = (j >= c) ? ld_cg(Ah + (int64_t)(b * IB + j) * NB + b * IB + c) : 0.0;
                 }
                 __syncthreads();
-                factor_block<NB, IB, false>(X, sf, b * IB);
+                if (factor_block<NB, IB, false>(X, sf, b * IB)) {
+                    restore();
+                    factor_block<NB, IB, false, true>(X, sf, b * IB);
+                }
             }
             TQR_PP(5);
             X.store(Ai + (int64_t)b * IB * NB, NB);

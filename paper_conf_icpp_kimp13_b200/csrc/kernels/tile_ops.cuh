@@ -370,27 +370,58 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
 }
 
 // ---------------------------------------------------------------- factor ib columns
-// X holds W = IB columns.  GEQRT mode (GE=true): column c's diagonal row is d = dbase + c,
-// rows < d are R (kept), rows > d become v (unit v_d implied, stored beta at row d).
-// TSQRT mode (GE=false): the top is sm.Rsm (IB x IB upper triangle, row c is R(dbase+c, :));
-// all NB rows of X are the dense V2 part.  On exit: X = reflectors, sm.tau, sm.Wsm = Gram V^T V;
-// build_T then forms the
-// IB x IB T factor as Tsm[i*LDT + c] = T(i, c) (upper triangle, zeros below).
-template <int NB, int IB, bool GE>
-__device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, IB, true>& sm, int dbase) {
+// Exact powers of two for the scaled norms of factor_block (reading Q26).
+// 2^e for -1022 <= e <= 1023, built from the exponent bits; 0 for e < -1022 (a contribution
+// scaled that far down is below the smallest normal relative to the column's largest entry).
+__device__ __forceinline__ double pow2s(int e) {
+    return e < -1022 ? 0.0 : __longlong_as_double((long long)(e + 1023) << 52);
+}
+// floor(log2 |x|) for normal x, -1022 for subnormal x, kNoExp for 0
+constexpr int kNoExp = -4096;
+__device__ __forceinline__ int exp2_floor(double x) {
+    const int f = (int)((__double_as_longlong(x) >> 52) & 0x7ff);
+    return x == 0.0 ? kNoExp : (f == 0 ? 1 : f) - 1023;
+}
+
+// SCALED = false (fast path): unscaled sums; returns true -- before touching sm.Rsm or building
+// the Gram -- when some column left the range where they are exact (an entry of the block above
+// 2^490, or a sub-column norm outside [2^-100, 2^100]); the caller then restores X and calls the
+// SCALED = true version, which scales every column as described below and never fails.
+template <int NB, int IB, bool GE, bool SCALED = false>
+__device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, IB, true>& sm, int dbase) {
     using G = Geom<NB, IB, IB>;
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW + 2 * t;   // row of acc[.][nf][e] = rbase + nf*8 + e
+    bool bad = false;
+    double wmax = 0.0;                      // fast path: largest |entry| of the block (incl. the TS top)
+    if constexpr (!SCALED) {
+#pragma unroll
+        for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+            for (int nf = 0; nf < G::NF; ++nf)
+                wmax = fmax(wmax, fmax(fabs(X.acc[mf][nf][0]), fabs(X.acc[mf][nf][1])));
+        if (!GE)
+            for (int idx = lane; idx < IB * IB; idx += 32) wmax = fmax(wmax, fabs(sm.Rsm[idx]));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) wmax = fmax(wmax, __shfl_xor_sync(0xffffffffu, wmax, o));
+    }
     // One barrier per column: each warp publishes, for column c, the partial ||x_below||^2, the
     // unscaled dots x^T a_j of every column j of the block and (GEQRT) the row-d entries a_dj;
     // after the barrier every thread forms beta, tau, scale = 1/(x0 - beta) and
     // w_j = a_dj (GEQRT) or R(c, j) (TSQRT) + scale * sum_w (x^T a_j)_w itself (v = scale x).
-    constexpr int FBW = 2 * IB + 2;          // per-warp record: dots[IB], diag row[IB], ||x||^2
+    constexpr int FBW = 2 * IB + 2;          // per-warp record: dots[IB], diag row[IB], ||x||^2, exponent
     double* fb = sm.red;                      // [2][kWarps][FBW] (double-buffered by column parity)
     double* Rout = sm.topsm;                  // TSQRT: R rows written as they are finished
     static_assert(2 * kWarps * FBW <= Smem<NB, IB, IB, true>::REDN, "factor record buffer");
     static_assert(IB * IB <= IB * G::LDW, "Rout buffer");
     TQR_FP0();
+    // Scaled norms and dots (dlarfg / dnrm2 semantics, reading Q26) at no extra barrier: each warp
+    // scales its part of x by the exact power of two 2^-e_w of its own largest |x| before forming
+    // ||x_w||^2 and x_w^T a_j, and records e_w; after the barrier the partials are brought to the
+    // column's common scale 2^-e, e = max(e_w, e(x0)), by exact power-of-two factors.  Nothing can
+    // overflow (scaled |x| < 2) and nothing that matters can underflow (a term is lost only when it
+    // is below 2^-1022 relative to the column's largest entry).  Powers of two are exact, so in the
+    // normal range every quantity is bitwise the unscaled formula's.
 
 #pragma unroll
     for (int mfc = 0; mfc < G::MF; ++mfc) {
@@ -399,7 +430,8 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             const int c = mfc * 8 + gc;
             const int d = dbase + c;
             double* fbp = fb + (c & 1) * (kWarps * FBW);
-            // 1. x = column c on my rows (from the lane holding it, same t), masked to rows > d (GEQRT)
+            // 1. x = column c on my rows (from the lane holding it, same t), masked to rows > d (GEQRT),
+            //    scaled by 2^-ew (ew = exponent of the warp's largest |x|)
             double xv[G::NF][2];
 #pragma unroll
             for (int nf = 0; nf < G::NF; ++nf)
@@ -409,6 +441,22 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                     const int r = rbase + nf * 8 + e;
                     xv[nf][e] = (!GE || r > d) ? x : 0.0;
                 }
+            int ew = 0;
+            if constexpr (SCALED) {
+                double xm = 0.0;
+#pragma unroll
+                for (int nf = 0; nf < G::NF; ++nf) xm = fmax(xm, fmax(fabs(xv[nf][0]), fabs(xv[nf][1])));
+                xm = fmax(xm, __shfl_xor_sync(0xffffffffu, xm, 1));
+                xm = fmax(xm, __shfl_xor_sync(0xffffffffu, xm, 2));
+                ew = exp2_floor(xm);
+                const int eu = (ew == kNoExp) ? 0 : ew;                   // x == 0 on this warp: unscaled
+                const double sw = pow2s(-eu / 2) * pow2s(eu / 2 - eu);   // 2^-ew in two exact factors
+#pragma unroll
+                for (int nf = 0; nf < G::NF; ++nf) {
+                    xv[nf][0] *= sw;
+                    xv[nf][1] *= sw;
+                }
+            }
             double ss = 0.0;
             if (g == 0) {
 #pragma unroll
@@ -444,25 +492,68 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                     rec[mf * 8 + g] = pd[mf];
                     if (GE) rec[IB + mf * 8 + g] = p0[mf];
                 }
-                if (g == 0) rec[2 * IB] = ss;
+                if (g == 0) {
+                    rec[2 * IB] = ss;
+                    if (SCALED) rec[2 * IB + 1] = (double)ew;
+                    else if (c == 0) rec[2 * IB + 1] = wmax;
+                }
             }
             __syncthreads();
-            // 2. reflector (dlarfg convention, readings Q1/Q4): beta = -sgn(x0) ||(x0, x)||
-            double xn2 = 0.0, x0 = 0.0;
+            // 2. reflector (dlarfg convention, readings Q1/Q4): beta = -sgn(x0) ||(x0, x)||, in units
+            //    of 2^ec; fw[w] = 2^(e_w - ec) brings warp w's partials to that scale
+            double x0 = 0.0, xn2 = 0.0, fw[kWarps];
+            int ec = 0;
+            if constexpr (SCALED) {
+                int ewv[kWarps];
+                ec = kNoExp;
 #pragma unroll
-            for (int w = 0; w < kWarps; ++w) {
-                xn2 += fbp[w * FBW + 2 * IB];
-                if (GE) x0 += fbp[w * FBW + IB + c];
+                for (int w = 0; w < kWarps; ++w) {
+                    ewv[w] = (int)fbp[w * FBW + 2 * IB + 1];
+                    ec = max(ec, ewv[w]);
+                    if (GE) x0 += fbp[w * FBW + IB + c];
+                }
+                if (!GE) x0 = sm.Rsm[c * IB + c];
+                ec = max(ec, exp2_floor(x0));
+                if (ec == kNoExp) ec = 0;                                 // x == 0 and x0 == 0
+#pragma unroll
+                for (int w = 0; w < kWarps; ++w) {
+                    fw[w] = pow2s(ewv[w] - ec);
+                    xn2 += fbp[w * FBW + 2 * IB] * (fw[w] * fw[w]);
+                }
+            } else {
+#pragma unroll
+                for (int w = 0; w < kWarps; ++w) {
+                    fw[w] = 1.0;
+                    xn2 += fbp[w * FBW + 2 * IB];
+                    if (GE) x0 += fbp[w * FBW + IB + c];
+                }
+                if (!GE) x0 = sm.Rsm[c * IB + c];
+                if (c == 0) {
+                    double bm = 0.0;
+#pragma unroll
+                    for (int w = 0; w < kWarps; ++w) bm = fmax(bm, fbp[w * FBW + 2 * IB + 1]);
+                    bad = bad || !(bm <= 0x1p490);
+                }
+                // GEQRT's last tile column has no sub-column (legitimately x = 0, tau = 0)
+                if (!(GE && d == NB - 1)) bad = bad || !(xn2 >= 0x1p-200) || !(x0 * x0 + xn2 <= 0x1p200);
             }
-            if (!GE) x0 = sm.Rsm[c * IB + c];
+            const double se = SCALED ? pow2s(-ec / 2) * pow2s(ec / 2 - ec) : 1.0;   // 2^-ec
+            const double x0s = x0 * se;
             double beta = x0, tau = 0.0, scale = 0.0;
             if (xn2 > 0.0) {
-                const double nrm = sqrt(x0 * x0 + xn2);
-                beta = (x0 < 0.0) ? nrm : -nrm;          // beta = -sgn(x0) ||x||, sgn(0)=+1
-                tau = (beta - x0) / beta;                  // correctly rounded: tau ||v||^2 = 2 decides
-                scale = 1.0 / (x0 - beta);                 // the orthogonality of I - tau v v^T
+                const double nrm = sqrt(x0s * x0s + xn2);
+                const double bs = (x0s < 0.0) ? nrm : -nrm;   // beta = -sgn(x0) ||x||, sgn(0)=+1
+                tau = (bs - x0s) / bs;                         // correctly rounded: tau ||v||^2 = 2 decides
+                scale = 1.0 / (x0s - bs);                      // the orthogonality of I - tau v v^T
+                beta = SCALED ? bs * pow2s(ec / 2) * pow2s(ec - ec / 2) : bs;   // back to the caller's scale
             }
-            // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = scale x (+ e_d)
+            // v on my rows = (x 2^-ew) 2^(ew - ec) scale (+ e_d); |v| <= 1
+            double vfac = scale;
+            if constexpr (SCALED) {
+#pragma unroll
+                for (int w = 0; w < kWarps; ++w) vfac = (w == wq) ? scale * fw[w] : vfac;
+            }
+            // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = x / (x0 - beta) (+ e_d)
             double tw[G::MF];
 #pragma unroll
             for (int mf = mfc; mf < G::MF; ++mf) {
@@ -472,7 +563,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                     double dsum = 0.0, base = 0.0;
 #pragma unroll
                     for (int w = 0; w < kWarps; ++w) {
-                        dsum += fbp[w * FBW + j];
+                        dsum += fbp[w * FBW + j] * fw[w];
                         if (GE) base += fbp[w * FBW + IB + j];
                     }
                     if (!GE) base = sm.Rsm[c * IB + j];
@@ -487,7 +578,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 for (int nf = 0; nf < G::NF; ++nf)
 #pragma unroll
                     for (int e = 0; e < 2; ++e) {
-                        const double v = scale * xv[nf][e] + ((GE && rbase + nf * 8 + e == d) ? 1.0 : 0.0);
+                        const double v = vfac * xv[nf][e] + ((GE && rbase + nf * 8 + e == d) ? 1.0 : 0.0);
                         X.acc[mf][nf][e] -= tw[mf] * v;
                     }
             }
@@ -498,7 +589,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
 #pragma unroll
                     for (int e = 0; e < 2; ++e) {
                         const int r = rbase + nf * 8 + e;
-                        if (!GE || r > d) X.acc[mfc][nf][e] *= scale;
+                        if (!GE || r > d) X.acc[mfc][nf][e] = vfac * xv[nf][e];
                         else if (r == d) X.acc[mfc][nf][e] = beta;
                     }
             }
@@ -507,6 +598,10 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 if (!GE) Rout[c * IB + c] = beta;
             }
         }
+    }
+    if (!SCALED && bad) {                   // CTA-uniform: sm.Rsm untouched, the caller redoes the block
+        __syncthreads();
+        return true;
     }
     if (!GE) {   // finished R rows -> Rsm (upper triangle)
         __syncthreads();
@@ -565,6 +660,7 @@ __device__ __forceinline__ void factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
         TQR_FP(1);
         // Gram in sm.Wsm; T is built by build_T (after the caller has stored X, freeing registers)
     }
+    return false;
 }
 
 // Forward dlarft recurrence T(c,c) = tau_c, T(0:c, c) = -tau_c T(0:c, 0:c) G(0:c, c), one row per

@@ -78,13 +78,48 @@ struct Owner {
     std::vector<std::vector<cudaEvent_t>> ev_u;     // ev_u[u][k]: stream u finished its step-k updates
     std::vector<std::vector<cudaEvent_t>> tm0, tm1; // profiling pairs per (u, k)
     std::vector<cudaEvent_t> tp0, tp1, tref;        // panel pairs, reference
+    std::vector<cudaEvent_t> tb0, tb1;              // transfer pairs per step (stats[3])
+    cudaEvent_t tl[4] = {nullptr, nullptr, nullptr, nullptr};   // layout pairs: load, store (stats[2])
     std::vector<std::vector<char>> tm_used;
-    std::vector<char> tp_used;
+    std::vector<char> tp_used, tb_used;
 };
 
 struct KStat {
     int64_t count = 0;
     double ms = 0.0, flops = 0.0;
+};
+
+// ---- CUDA-IPC transport (tqr_options.transport = TQR_TRANSPORT_IPC)
+// Export blob of one rank: IPC handles of the allocations peers touch.
+enum IpcSlot {
+    H_FLAGS = 0,
+    H_RB = 1,        // receive slots: H_RB + 5*s + {tiles, T, V, M, MT}
+    H_TILES = 11, H_VIMG, H_T, H_VEXP, H_MIMG, H_MT,   // reflector storage (apply/solve replication)
+    H_RSSEND,        // row split: this rank's R_g for the stage-2 gather
+    kNH
+};
+struct IpcBlob {
+    uint32_t magic;
+    int32_t rank, dev, world;
+    uint64_t present;            // bit i: handle i exported
+    cudaIpcMemHandle_t h[kNH];
+};
+constexpr uint32_t kIpcMagic = 0x54515231u;   // "TQR1"
+// 64-bit flags in each rank's flag block (waits are always on the waiter's own block):
+constexpr int F_READY = 0;       // [slot]            panel of step k landed in my receive slot k%2 (root writes)
+constexpr int F_FREED = 8;       // [2*src + slot]    rank src's slot is free for step k (src writes into root's block)
+constexpr int F_DONE = 160;      // [src]             rank src finished factorization #E (its storage is final)
+constexpr int F_APPLIED = 224;   // [src]             rank src finished apply/solve call #seq (its pulls)
+constexpr int F_RSREADY = 288;   // [src]             row split: rank src's R_g is in its rs_send (rank 0's block)
+constexpr int F_PULLED = 352;    //                   row split: rank 0 has pulled my R_g of #E (my block)
+constexpr int kFlagWords = 512;
+constexpr int kIpcMaxWorld = 64;
+struct IpcPeer {
+    int dev = -1;
+    uint64_t* flags = nullptr;
+    void* rb[2][5] = {{nullptr}};   // receive slot s: tiles, T, V, M, MT
+    void* st[6] = {nullptr};        // tiles, Vimg, T, Vexp, Mimg, MT
+    void* rs_send = nullptr;
 };
 
 }  // namespace
@@ -153,7 +188,20 @@ struct tqr_plan_s {
     cudaStream_t rs_stream = nullptr;       // this process's gather stream
 
     bool nccl_mode = false;         // one process per GPU, panels broadcast with NCCL
-    bool multiproc() const { return nccl_mode; }
+    bool ipc_mode = false;          // one process per owner, panels copied into CUDA-IPC-mapped slots
+    bool ipc_connected = false;
+    uint64_t* flags64 = nullptr;    // this rank's IPC flag block (kFlagWords)
+    std::vector<IpcPeer> peers;     // IPC: world entries (own entry = local pointers)
+    std::vector<void*> ipc_opened;  // peer mappings to close
+    uint64_t apply_seq = 0;         // IPC apply/solve collectives so far
+    uint64_t fact_id = 0;           // flag value of the last completed factorization
+    uint64_t rs_epoch = 0;          // row split factorizations so far
+    // multi-owner apply / solve: single-owner replica of the factorization on this device
+    tqr_plan rep = nullptr;
+    uint64_t fact_gen = 0, rep_gen = 0;
+    // issued-op trace of the last tqr_factor_tiles (tqr_issued_ops)
+    std::vector<int32_t> issued;
+    bool multiproc() const { return nccl_mode || ipc_mode; }
     bool f32() const { return dtype == TQR_F32; }
     // p + e elements
     template <class E = void>
@@ -221,8 +269,10 @@ void free_owner(Owner& o) {
     F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp); F(o.Mimg); F(o.MT); F(o.Mt);
     for (int s = 0; s < 2; ++s) { F(o.rb_M[s]); F(o.rb_MT[s]); }
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
-    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref, &o.ev_load, &o.ev_chunk, &o.ev_dom})
+    for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref, &o.ev_load, &o.ev_chunk, &o.ev_dom,
+                    &o.tb0, &o.tb1})
         for (auto e : *v) if (e) cudaEventDestroy(e);
+    for (auto e : o.tl) if (e) cudaEventDestroy(e);
     for (auto* vv : {&o.ev_u, &o.tm0, &o.tm1})
         for (auto& v : *vv) for (auto e : v) if (e) cudaEventDestroy(e);
     for (auto s : o.s_u) if (s) cudaStreamDestroy(s);
@@ -234,13 +284,14 @@ void free_owner(Owner& o) {
 }
 
 // Host-side DAG (Fig. 3) per rank, the same order the executor issues.
+// rank < 0: every owner is local (in-process plan) -> all owners' records.
 void build_schedule(int64_t q, const std::vector<int32_t>& owner_of, int rank, std::vector<int32_t>& out) {
     for (int k = 0; k < q; ++k) {
         const int o = owner_of[k];
-        if (o == rank) { out.insert(out.end(), {0, k, k, k, o}); }
+        if (rank < 0 || o == rank) { out.insert(out.end(), {0, k, k, k, o}); }
         out.insert(out.end(), {1, k, k, k, o});
         for (int j = k + 1; j < q; ++j)
-            if (owner_of[j] == rank) out.insert(out.end(), {2, k, k, j, o});
+            if (rank < 0 || owner_of[j] == rank) out.insert(out.end(), {2, k, k, j, o});
     }
 }
 
@@ -396,9 +447,21 @@ tqr_status tqr_create(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dt
     return tqr_create_ex(m, n, nb, ib, dtype, ndev, guide, guide_len, nullptr, out);
 }
 
+static void ipc_release(tqr_plan h) {
+    for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
+    h->ipc_opened.clear();
+    h->peers.clear();
+    if (h->flags64) cudaFree(h->flags64);
+    h->flags64 = nullptr;
+    if (h->rep) { tqr_destroy(h->rep); h->rep = nullptr; }
+    cudaGetLastError();
+}
+
 tqr_status tqr_destroy(tqr_plan h) {
     if (!h) return TQR_OK;
     if (h->rs) {
+        if (h->rs_stream) cudaStreamSynchronize(h->rs_stream);
+        ipc_release(h);
         for (size_t i = 0; i < h->kids.size(); ++i) {
             cudaSetDevice(h->kid_dev[i]);
             tqr_destroy(h->kids[i]);
@@ -423,6 +486,7 @@ tqr_status tqr_destroy(tqr_plan h) {
     }
     if (h->comm && h->nccl) h->nccl->CommDestroy(h->comm);
     if (!h->owners.empty()) cudaSetDevice(h->owners[0].dev);
+    ipc_release(h);
     if (h->bw) cudaFree(h->bw);
     if (h->dflag) cudaFree(h->dflag);
     if (h->prog) cudaFree(h->prog);
@@ -445,7 +509,8 @@ tqr_status tqr_row_split_ranges(int64_t m, int32_t nb, int32_t ndev, int64_t* r0
 
 // Row-split plan (see tqr_options.row_split): owner g holds tile rows [g p / G, (g+1) p / G).
 static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
-                                   const tqr_options& o, bool use_nccl, int world, tqr_plan* out) {
+                                   const tqr_options& o, bool mp, bool use_ipc, int world, tqr_plan* out) {
+    const bool use_nccl = mp && !use_ipc;
     const int64_t p = (m + nb - 1) / nb;
     if (n > nb) return fail(nullptr, TQR_ERR_UNSUPPORTED, "row split: a single column tile (n <= nb) only");
     tqr_plan h = new tqr_plan_s();
@@ -454,9 +519,10 @@ static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib,
     h->dtype = dtype; h->ndev = ndev; h->es = (dtype == TQR_F32) ? 4 : 8;
     h->guide.assign(1, 0);
     h->owner_of.assign(1, 0);
-    h->rank = use_nccl ? o.rank : 0;
+    h->rank = mp ? o.rank : 0;
     h->world = world;
     h->nccl_mode = use_nccl;
+    h->ipc_mode = use_ipc;
     h->profile = o.profile != 0;
     auto bail = [&](tqr_status st) { std::string e = h->err; tqr_destroy(h); g_create_error = e; return st; };
     h->rs_r0.resize(ndev);
@@ -474,8 +540,8 @@ static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib,
     co.tree_group = o.tree_group;
     co.row_split = -1;
     for (int g = 0; g < ndev; ++g) {
-        if (use_nccl && g != h->rank) continue;
-        const int dev = (use_nccl || o.logical_devices) ? cur : g;
+        if (mp && g != h->rank) continue;
+        const int dev = (mp || o.logical_devices) ? cur : g;
         if (cudaSetDevice(dev) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "cudaSetDevice(%d)", dev));
         tqr_plan kid = nullptr;
         tqr_status st = tqr_create_ex(h->rs_rows[g], n, nb, ib, dtype, 1, nullptr, 0, &co, &kid);
@@ -496,13 +562,18 @@ static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib,
             if (cudaMalloc(&h->stk, (size_t)h->es * ndev * nb * n) != cudaSuccess)
                 return bail(fail(h, TQR_ERR_ALLOC, "row split: stacked R buffer"));
         }
-        if (use_nccl) {
+        if (mp) {
             if (cudaMalloc(&h->rs_send, (size_t)h->es * nb * n) != cudaSuccess ||
-                cudaMalloc(&h->rs_recv, (size_t)h->es * ndev * nb * n) != cudaSuccess)
+                (use_nccl && cudaMalloc(&h->rs_recv, (size_t)h->es * ndev * nb * n) != cudaSuccess))
                 return bail(fail(h, TQR_ERR_ALLOC, "row split: gather buffers"));
         }
     }
-    cudaSetDevice(use_nccl || o.logical_devices ? cur : 0);
+    if (use_ipc) {
+        if (cudaMalloc(&h->flags64, kFlagWords * sizeof(uint64_t)) != cudaSuccess ||
+            cudaMemset(h->flags64, 0, kFlagWords * sizeof(uint64_t)) != cudaSuccess)
+            return bail(fail(h, TQR_ERR_ALLOC, "IPC flag block"));
+    }
+    cudaSetDevice(mp || o.logical_devices ? cur : 0);
     if (cudaStreamCreateWithFlags(&h->rs_stream, cudaStreamNonBlocking) != cudaSuccess)
         return bail(fail(h, TQR_ERR_CUDA, "row split: stream"));
     if (use_nccl) {
@@ -534,23 +605,30 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     tqr_options o{};
     if (opt) o = *opt;
     // NCCL mode: world > 1, or a single-rank communicator when an nccl_id is given explicitly
-    const bool use_nccl = o.world > 1 || o.nccl_id != nullptr;
+    // Multi-process: world > 1, a 1-rank NCCL communicator (nccl_id), or an explicit IPC transport.
+    if (o.transport < TQR_TRANSPORT_AUTO || o.transport > TQR_TRANSPORT_IPC)
+        return fail(nullptr, TQR_ERR_ARG, "unknown transport %d", o.transport);
+    const bool mp = o.world > 1 || o.nccl_id != nullptr || o.transport == TQR_TRANSPORT_IPC;
+    const bool use_ipc = mp && (o.transport == TQR_TRANSPORT_IPC || (o.transport == TQR_TRANSPORT_AUTO && !o.nccl_id));
+    const bool use_nccl = mp && !use_ipc;
     const int world = o.world > 1 ? o.world : 1;
-    if (use_nccl && (o.rank < 0 || o.rank >= world || ndev != world || !o.nccl_id))
-        return fail(nullptr, TQR_ERR_ARG, "multi-process: need 0 <= rank < world == ndev and nccl_id");
+    if (mp && (o.rank < 0 || o.rank >= world || ndev != world))
+        return fail(nullptr, TQR_ERR_ARG, "multi-process: need 0 <= rank < world == ndev");
+    if (use_nccl && !o.nccl_id) return fail(nullptr, TQR_ERR_ARG, "NCCL transport: nccl_id is required");
+    if (use_ipc && world > kIpcMaxWorld) return fail(nullptr, TQR_ERR_ARG, "IPC transport: world > %d", kIpcMaxWorld);
     int ndevices = 0;
     if (cudaGetDeviceCount(&ndevices) != cudaSuccess || ndevices < 1) {
         cudaGetLastError();
         return fail(nullptr, TQR_ERR_CUDA, "no CUDA device");
     }
-    if (!use_nccl && !o.logical_devices && ndev > ndevices)
+    if (!mp && !o.logical_devices && ndev > ndevices)
         return fail(nullptr, TQR_ERR_ARG, "ndev %d > %d visible CUDA devices (set logical_devices)", ndev, ndevices);
 
     {
         const int64_t pp = (m + nb - 1) / nb, qq = (n + nb - 1) / nb;
         const bool rs = o.row_split > 0 ||
                         (o.row_split == 0 && qq == 1 && ndev > 1 && dtype == TQR_F64 && pp >= 2 * ndev);
-        if (rs) return create_row_split(m, n, nb, ib, dtype, ndev, o, use_nccl, world, out);
+        if (rs) return create_row_split(m, n, nb, ib, dtype, ndev, o, mp, use_ipc, world, out);
     }
     tqr_plan h = new tqr_plan_s();
     h->m = m; h->n = n; h->nb = nb; h->ib = ib; h->p = (int)((m + nb - 1) / nb); h->q = (int)((n + nb - 1) / nb);
@@ -558,9 +636,10 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     h->es = (dtype == TQR_F32) ? 4 : 8;
     h->vt = (dtype == TQR_F32) ? tqr::f32_img_tile(nb, ib) : (int64_t)nb * nb;
     h->logical = o.logical_devices != 0;
-    h->rank = use_nccl ? o.rank : 0;
+    h->rank = mp ? o.rank : 0;
     h->world = world;
     h->nccl_mode = use_nccl;
+    h->ipc_mode = use_ipc;
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_LA_OVERLAP")) h->la_overlap = atoi(e) != 0;
@@ -605,7 +684,9 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     }
     // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
     // panel is on the critical path (few trailing columns per panel step or several owners).
-    h->panel_split = (h->q <= 4) ? 4 : 2;   // measured: 4 for tall / few columns, 2 otherwise
+    // measured (r02): 4 sub-slices (W = 8) cut the C5 8-owner critical path 417 -> 345 ms and C3
+    // 236.9 -> 232.1 ms; the last column blocks' sequential applies bound the TS wavefront
+    h->panel_split = 4;
     if (ib < 32 && h->panel_split > 2) h->panel_split = 2;
     if (const char* e = getenv("TQR_PANEL_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->panel_split = v; }
     if (ib / h->panel_split < 8) h->panel_split = 1;
@@ -614,7 +695,7 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
 
     int cur = 0;
     cudaGetDevice(&cur);
-    const int nown = use_nccl ? 1 : ndev;
+    const int nown = mp ? 1 : ndev;
     h->owners.resize(nown);
     auto bail = [&](tqr_status s) { std::string e = h->err; tqr_destroy(h); g_create_error = e; return s; };
     int prio_lo = 0, prio_hi = 0;
@@ -622,8 +703,8 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     const int64_t p = h->p, tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb;
     for (int li = 0; li < nown; ++li) {
         Owner& ow = h->owners[li];
-        ow.id = use_nccl ? h->rank : li;
-        ow.dev = (use_nccl || h->logical) ? cur : li;
+        ow.id = mp ? h->rank : li;
+        ow.dev = (mp || h->logical) ? cur : li;
         ow.lidx.assign(h->q, -1);
         for (int j = 0; j < h->q; ++j)
             if (h->owner_of[j] == ow.id) { ow.lidx[j] = (int32_t)ow.cols.size(); ow.cols.push_back(j); }
@@ -650,8 +731,11 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         if (ok && h->profile) {
             ow.tm0.resize(S); ow.tm1.resize(S); ow.tm_used.assign(S, std::vector<char>(h->q, 0));
             for (int u = 0; u < S && ok; ++u) ok = mkev(ow.tm0[u], h->q, true) && mkev(ow.tm1[u], h->q, true);
-            ok = ok && mkev(ow.tp0, h->q, true) && mkev(ow.tp1, h->q, true) && mkev(ow.tref, 1, true);
+            ok = ok && mkev(ow.tp0, h->q, true) && mkev(ow.tp1, h->q, true) && mkev(ow.tref, 1, true) &&
+                 mkev(ow.tb0, h->q, true) && mkev(ow.tb1, h->q, true);
+            for (auto& e : ow.tl) ok = ok && cudaEventCreate(&e) == cudaSuccess;
             ow.tp_used.assign(h->q, 0);
+            ow.tb_used.assign(h->q, 0);
         }
         if (!ok) return bail(fail(h, TQR_ERR_CUDA, "event creation failed"));
         const size_t nc = ow.cols.size();
@@ -701,7 +785,13 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
         }
     }
     // peer access between physical owners (single-process, several GPUs)
-    if (!use_nccl && !h->logical && ndev > 1) {
+    if (use_ipc) {
+        cudaSetDevice(cur);
+        if (cudaMalloc(&h->flags64, kFlagWords * sizeof(uint64_t)) != cudaSuccess ||
+            cudaMemset(h->flags64, 0, kFlagWords * sizeof(uint64_t)) != cudaSuccess)
+            return bail(fail(h, TQR_ERR_ALLOC, "IPC flag block"));
+    }
+    if (!mp && !h->logical && ndev > 1) {
         for (int a = 0; a < ndev; ++a)
             for (int b = 0; b < ndev; ++b) {
                 if (a == b) continue;
@@ -723,6 +813,132 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     cudaSetDevice(cur);
     *out = h;
     return TQR_OK;
+}
+
+// ------------------------------------------------------------------ CUDA-IPC transport handshake
+namespace {
+int plan_device(tqr_plan h) {
+    if (!h->owners.empty()) return h->owners[0].dev;
+    if (!h->kid_dev.empty()) return h->kid_dev[0];
+    int d = 0;
+    cudaGetDevice(&d);
+    return d;
+}
+cudaStream_t plan_comm_stream(tqr_plan h) { return h->rs ? h->rs_stream : h->owners[0].s_comm; }
+// pointers a peer needs, in IpcSlot order (null = not allocated on this rank)
+void export_ptrs(tqr_plan h, void* out[kNH]) {
+    for (int i = 0; i < kNH; ++i) out[i] = nullptr;
+    out[H_FLAGS] = h->flags64;
+    if (h->rs) {
+        out[H_RSSEND] = h->rs_send;
+        return;
+    }
+    Owner& o = h->owners[0];
+    for (int sl = 0; sl < 2; ++sl) {
+        out[H_RB + 5 * sl + 0] = o.rb_tiles[sl];
+        out[H_RB + 5 * sl + 1] = o.rb_T[sl];
+        out[H_RB + 5 * sl + 2] = o.rb_V[sl];
+        out[H_RB + 5 * sl + 3] = o.rb_M[sl];
+        out[H_RB + 5 * sl + 4] = o.rb_MT[sl];
+    }
+    out[H_TILES] = o.tiles; out[H_VIMG] = o.Vimg; out[H_T] = o.T; out[H_VEXP] = o.Vexp;
+    out[H_MIMG] = o.Mimg; out[H_MT] = o.MT;
+}
+void peer_from_ptrs(IpcPeer& pr, void* const ptr[kNH]) {
+    pr.flags = static_cast<uint64_t*>(ptr[H_FLAGS]);
+    for (int sl = 0; sl < 2; ++sl)
+        for (int f = 0; f < 5; ++f) pr.rb[sl][f] = ptr[H_RB + 5 * sl + f];
+    for (int f = 0; f < 6; ++f) pr.st[f] = ptr[H_TILES + f];
+    pr.rs_send = ptr[H_RSSEND];
+}
+}  // namespace
+
+tqr_status tqr_ipc_handle(tqr_plan h, void* buf, int64_t cap, int64_t* len) {
+    if (!h || !len) return fail(h, TQR_ERR_ARG, "ipc_handle: bad arguments");
+    if (!h->ipc_mode) return fail(h, TQR_ERR_STATE, "ipc_handle: the plan does not use the IPC transport");
+    *len = (int64_t)sizeof(IpcBlob);
+    if (!buf) return TQR_OK;
+    if (cap < *len) return fail(h, TQR_ERR_ARG, "ipc_handle: capacity %lld < %lld", (long long)cap, (long long)*len);
+    IpcBlob b;
+    std::memset(&b, 0, sizeof(b));
+    b.magic = kIpcMagic;
+    b.rank = h->rank;
+    b.world = h->world;
+    b.dev = plan_device(h);
+    void* ptr[kNH];
+    export_ptrs(h, ptr);
+    CUDA_TRY(h, cudaSetDevice(b.dev));
+    for (int i = 0; i < kNH; ++i)
+        if (ptr[i]) {
+            CUDA_TRY(h, cudaIpcGetMemHandle(&b.h[i], ptr[i]));
+            b.present |= 1ull << i;
+        }
+    std::memcpy(buf, &b, sizeof(b));
+    return TQR_OK;
+}
+
+tqr_status tqr_ipc_connect(tqr_plan h, const void* all, int64_t len) {
+    if (!h || !all) return fail(h, TQR_ERR_ARG, "ipc_connect: bad arguments");
+    if (!h->ipc_mode) return fail(h, TQR_ERR_STATE, "ipc_connect: the plan does not use the IPC transport");
+    if (h->ipc_connected) return fail(h, TQR_ERR_STATE, "ipc_connect: already connected");
+    const int64_t bs = (int64_t)sizeof(IpcBlob);
+    if (len != bs * h->world) return fail(h, TQR_ERR_ARG, "ipc_connect: %lld bytes, expected %lld", (long long)len, (long long)(bs * h->world));
+    const int dev = plan_device(h);
+    CUDA_TRY(h, cudaSetDevice(dev));
+    h->peers.assign(h->world, IpcPeer());
+    for (int r = 0; r < h->world; ++r) {
+        IpcBlob b;
+        std::memcpy(&b, static_cast<const char*>(all) + r * bs, sizeof(b));
+        if (b.magic != kIpcMagic || b.rank != r || b.world != h->world)
+            return fail(h, TQR_ERR_ARG, "ipc_connect: blob %d is not rank %d's export", r, r);
+        void* ptr[kNH];
+        if (r == h->rank) {
+            export_ptrs(h, ptr);
+        } else {
+            for (int i = 0; i < kNH; ++i) {
+                ptr[i] = nullptr;
+                if (b.present >> i & 1ull) {
+                    CUDA_TRY(h, cudaIpcOpenMemHandle(&ptr[i], b.h[i], cudaIpcMemLazyEnablePeerAccess));
+                    h->ipc_opened.push_back(ptr[i]);
+                }
+            }
+        }
+        peer_from_ptrs(h->peers[r], ptr);
+        h->peers[r].dev = b.dev;
+    }
+    // arm: my receive slots 0 / 1 are free for steps 0 / 1 of the first factorization, at every
+    // possible root (the flag lives in the root's block; roots only ever wait on their own block)
+    cudaStream_t s = plan_comm_stream(h);
+    for (int d = 0; d < h->world; ++d) {
+        if (d == h->rank) continue;
+        for (int sl = 0; sl < 2; ++sl)
+            CUDA_TRY(h, tqr::sig_write(s, h->peers[d].flags + F_FREED + 2 * h->rank + sl, (uint64_t)h->epoch + 1 + sl));
+    }
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    h->ipc_connected = true;
+    return TQR_OK;
+}
+
+tqr_status tqr_issued_ops(tqr_plan h, int32_t* ops, int64_t cap, int64_t* count) {
+    if (!h || !count) return fail(h, TQR_ERR_ARG, "issued_ops: bad arguments");
+    *count = (int64_t)h->issued.size() / 5;
+    if (ops) {
+        if (cap < *count) return fail(h, TQR_ERR_ARG, "issued_ops: capacity %lld < %lld", (long long)cap, (long long)*count);
+        std::copy(h->issued.begin(), h->issued.end(), ops);
+    }
+    return TQR_OK;
+}
+
+int32_t tqr_plan_flags(tqr_plan h) {
+    if (!h) return 0;
+    int32_t f = 0;
+    if (h->rs) f |= TQR_PLAN_ROW_SPLIT;
+    if (h->tree_L > 0 || (h->rs && !h->kids.empty() && h->kids[0]->tree_L > 0)) f |= TQR_PLAN_TREE;
+    if (h->multiproc()) f |= TQR_PLAN_MULTIPROC;
+    if (h->ipc_mode) f |= TQR_PLAN_IPC;
+    if (h->nccl_mode) f |= TQR_PLAN_NCCL;
+    if (h->f32()) f |= TQR_PLAN_F32;
+    return f;
 }
 
 int32_t tqr_owner(tqr_plan h, int64_t j) {
@@ -907,6 +1123,7 @@ tqr_status rs_load(tqr_plan h, const void* A, int64_t lda) {
 // every owner factors its row block; the owners' R factors (tile 0 of each block) are stacked on
 // owner 0 (peer copies, or an NCCL all-gather) with their reflectors zeroed, and factored again
 tqr_status rs_factor(tqr_plan h) {
+    if (h->ipc_mode && !h->ipc_connected) return fail(h, TQR_ERR_STATE, "IPC plan not connected (tqr_ipc_connect)");
     const int G = h->ndev, nb = h->nb;
     const int64_t n = h->n, es = h->es, ld = (int64_t)G * nb;
     for (size_t i = 0; i < h->kids.size(); ++i) {
@@ -914,7 +1131,25 @@ tqr_status rs_factor(tqr_plan h) {
         tqr_status st = tqr_factor_tiles(h->kids[i]);
         if (st) return kid_fail(h, h->kids[i], st);
     }
-    if (h->multiproc()) {
+    if (h->ipc_mode) {
+        // every rank publishes its R_g (tile 0 of its block) in rs_send once rank 0 has pulled the
+        // previous one; rank 0 pulls all of them into the stack (IPC reads), then releases rs_send
+        const uint64_t E = ++h->rs_epoch;
+        tqr_plan kid = h->kids[0];
+        CUDA_TRY(h, cudaSetDevice(h->kid_dev[0]));
+        cudaStream_t s = h->rs_stream;
+        CUDA_TRY(h, tqr::sig_wait_geq(s, h->flags64 + F_PULLED, E - 1));
+        CUDA_TRY(h, cudaMemcpyAsync(h->rs_send, kid->owners[0].tiles, (size_t)es * nb * n, cudaMemcpyDeviceToDevice, s));
+        CUDA_TRY(h, tqr::sig_write(s, h->peers[0].flags + F_RSREADY + h->rank, E));
+        if (h->top) {
+            for (int g = 0; g < G; ++g) {
+                CUDA_TRY(h, tqr::sig_wait_geq(s, h->flags64 + F_RSREADY + g, E));
+                CUDA_TRY(h, cudaMemcpy2DAsync(h->at(h->stk, (int64_t)g * nb), ld * es, h->peers[g].rs_send, nb * es,
+                                              nb * es, n, cudaMemcpyDefault, s));
+            }
+            for (int g = 0; g < G; ++g) CUDA_TRY(h, tqr::sig_write(s, h->peers[g].flags + F_PULLED, E));
+        }
+    } else if (h->multiproc()) {
         tqr_plan kid = h->kids[0];
         CUDA_TRY(h, cudaSetDevice(h->kid_dev[0]));
         CUDA_TRY(h, cudaMemcpyAsync(h->rs_send, kid->owners[0].tiles, (size_t)es * nb * n, cudaMemcpyDeviceToDevice,
@@ -972,6 +1207,28 @@ tqr_status rs_store(tqr_plan h, void* A, int64_t lda) {
 }  // namespace
 
 // ------------------------------------------------------------------ a1: load
+namespace {
+// stats[2]: the layout pass just completed (ev = 0: load, 2: store) on every owner: device time of
+// the slowest owner, algorithmic bytes = read + write of the owned columns (es * m * nb each way)
+tqr_status layout_stat(tqr_plan h, int ev) {
+    if (!h->profile) return TQR_OK;
+    float mx = 0.f;
+    double bytes = 0.0;
+    for (auto& o : h->owners) {
+        if (o.cols.empty()) continue;
+        CUDA_TRY(h, cudaSetDevice(o.dev));
+        float t = 0.f;
+        CUDA_TRY(h, cudaEventElapsedTime(&t, o.tl[ev], o.tl[ev + 1]));
+        mx = std::max(mx, t);
+        bytes += 2.0 * h->es * (double)h->m * h->nb * o.cols.size();
+    }
+    h->stats[2].count += 1;
+    h->stats[2].ms += mx;
+    h->stats[2].flops += bytes;
+    return TQR_OK;
+}
+}  // namespace
+
 tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
     if (!h) return TQR_ERR_ARG;
     if (h->rs) {
@@ -989,6 +1246,7 @@ tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, cudaSetDevice(o.dev));
         const int nc = (int)o.cols.size();
+        if (h->profile) CUDA_TRY(h, cudaEventRecord(o.tl[0], o.s_upd));
         if (pi.kind == Mem::Device && pi.dev == o.dev) {
             CUDA_TRY(h, to_tiles(h, A, lda, nb * lda, o.tiles, o.cols_dev, 0, nc, o.s_upd));
             h->launches++;
@@ -1005,8 +1263,11 @@ tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
             CUDA_TRY(h, to_tiles(h, o.io, h->m, h->m * nb, o.tiles, o.cols_dev, 1, nc, o.s_upd));
             h->launches++;
         }
+        if (h->profile) CUDA_TRY(h, cudaEventRecord(o.tl[1], o.s_upd));
     }
-    return sync_all(h);
+    tqr_status st = sync_all(h);
+    if (st) return st;
+    return layout_stat(h, 0);
 }
 
 // ------------------------------------------------------------------ a2-a7: factor
@@ -1105,6 +1366,7 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
 tqr_status tqr_factor_tiles(tqr_plan h) {
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
+    if (h->ipc_mode && !h->ipc_connected) return fail(h, TQR_ERR_STATE, "IPC plan not connected (tqr_ipc_connect)");
     if (h->rs) return rs_factor(h);
     const int p = h->p, q = h->q, nb = h->nb, ib = h->ib;
     // bulk-update streams: round-robin (column lc on stream lc % S) for resident data; a streamed
@@ -1113,8 +1375,11 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
     // stream's step-1 launch behind its last column's load)
     const int S = h->streamed ? h->nstreams_io : h->nstreams;
     const int64_t tile = (int64_t)nb * nb, tsz = (int64_t)ib * nb, colsz = (int64_t)p * tile, vt = h->vt;
+    const size_t es = h->es;
     const unsigned epoch0 = h->epoch;
     h->epoch += (unsigned)q + 1;
+    h->factored = false;
+    h->fact_gen += 1;
     // order all owner streams after whatever ran before (load, previous calls)
     for (auto& o : h->owners) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
@@ -1122,6 +1387,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
         if (h->profile) {
             for (auto& v : o.tm_used) std::fill(v.begin(), v.end(), 0);
             std::fill(o.tp_used.begin(), o.tp_used.end(), 0);
+            std::fill(o.tb_used.begin(), o.tb_used.end(), 0);
             CUDA_TRY(h, cudaEventRecord(o.tref[0], o.s_panel));
         }
     }
@@ -1132,11 +1398,27 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
         for (int u = 0; u < S; ++u) CUDA_TRY(h, cudaStreamWaitEvent(st, D.ev_u[u][kk], 0));
         return TQR_OK;
     };
-    for (int k = 0; k < q; ++k) {
+    // does rank / owner d hold a column > k (i.e. receive panel k)?
+    auto needs = [&](int d, int k) {
+        for (int j = k + 1; j < q; ++j) if (h->owner_of[j] == d) return true;
+        return false;
+    };
+    auto emit = [&](int op, int k, int i, int j, int root) { h->issued.insert(h->issued.end(), {op, k, i, j, root}); };
+    // The executor consumes the host-side DAG schedule (tqr_schedule: PANEL, BCAST, UPDATE records
+    // per step), all owners' records for an in-process plan, this rank's for a multi-process one.
+    std::vector<int32_t> sched;
+    build_schedule(q, h->owner_of, h->multiproc() ? h->rank : -1, sched);
+    h->issued.clear();
+    const size_t nrec = sched.size() / 5;
+    size_t pos = 0;
+    while (pos < nrec) {
+        const int op = sched[5 * pos], k = sched[5 * pos + 1];
         const int ok = h->owner_of[k];
         Owner* O = h->local(ok);
-        // ---- PANEL(k)
-        if (O) {
+        if (op == 0) {
+            // ---- PANEL(k)
+            ++pos;
+            if (!O) return fail(h, TQR_ERR_STATE, "schedule: PANEL(%d) of a remote owner", k);
             CUDA_TRY(h, cudaSetDevice(O->dev));
             if (k > 0 && !h->lookahead) { tqr_status st = wait_all_u(*O, O->s_panel, k - 1); if (st) return st; }
             if (h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(O->s_panel, O->ev_load[O->lidx[k]], 0));
@@ -1145,11 +1427,11 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             if (st) return st;
             if (h->profile) { CUDA_TRY(h, cudaEventRecord(O->tp1[k], O->s_panel)); O->tp_used[k] = 1; }
             CUDA_TRY(h, cudaEventRecord(O->ev_panel[k], O->s_panel));
+            emit(0, k, k, k, ok);
             if (h->streamed) {
                 // column k is final once PANEL(k) is done (later steps touch columns > k only, and
                 // updates read the reflectors from the stage images): a8 + D2H on the I/O stream
                 const int lc = O->lidx[k];
-                const size_t es = h->es;
                 void* slab = h->at(O->io, (int64_t)lc * h->m * nb);
                 CUDA_TRY(h, cudaStreamWaitEvent(O->s_io, O->ev_panel[k], 0));
                 CUDA_TRY(h, from_tiles(h, slab, h->m, h->m * nb, h->at(O->tiles, lc * colsz), O->cols_dev + lc, 1,
@@ -1159,64 +1441,126 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                                               cudaMemcpyDefault, O->s_io));
                 h->launches++;
             }
+            continue;
         }
-        // ---- BCAST(k): the reflector-tile images k..p-1, their T factors and the explicit V
-        if (h->multiproc()) {
-            Owner& R = h->owners[0];
-            CUDA_TRY(h, cudaSetDevice(R.dev));
+        if (op == 1) {
+            // ---- BCAST(k): the reflector-tile images k..p-1, their T factors and the explicit V
+            // (+ tree merge images / T) from owner(k) to every owner of a column > k
+            ++pos;
             const int slot = k & 1;
-            const bool root = (ok == h->rank);
-            if (root) CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_panel[k], 0));
-            if (!root && k >= 2) {
-                tqr_status st = wait_all_u(R, R.s_comm, k - 2);
-                if (st) return st;
-                CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
-            }
-            PanelRefs b = root ? own_refs(h, R, R.lidx[k]) : recv_refs(h, R, slot);
-            const ncclDataType_t dt = h->f32() ? ncclFloat32 : ncclFloat64;
-            void* bv = h->at(b.V, k * vt);
-            void* bt = h->at(b.T, k * tsz);
-            NCCL_TRY(h, h->nccl->GroupStart());
-            NCCL_TRY(h, h->nccl->Broadcast(bv, bv, (size_t)(p - k) * vt, dt, ok, h->comm, R.s_comm));
-            NCCL_TRY(h, h->nccl->Broadcast(bt, bt, (size_t)(p - k) * tsz, dt, ok, h->comm, R.s_comm));
-            NCCL_TRY(h, h->nccl->Broadcast(b.Vexp, b.Vexp, (size_t)vt, dt, ok, h->comm, R.s_comm));
-            if (h->ndom(k) > 1) {
-                const size_t D = h->ndom(k);
-                NCCL_TRY(h, h->nccl->Broadcast(b.M, b.M, D * vt, dt, ok, h->comm, R.s_comm));
-                NCCL_TRY(h, h->nccl->Broadcast(b.MT, b.MT, D * tsz, dt, ok, h->comm, R.s_comm));
-            }
-            NCCL_TRY(h, h->nccl->GroupEnd());
-            CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
-        } else {
-            for (auto& D : h->owners) {
-                if (D.id == ok) continue;
-                bool needs = false;
-                for (int32_t j : D.cols) if (j > k) { needs = true; break; }
-                if (!needs) continue;
-                CUDA_TRY(h, cudaSetDevice(D.dev));
-                const int slot = k & 1;
-                CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_panel[k], 0));
-                if (k >= 2) {
-                    tqr_status st = wait_all_u(D, D.s_comm, k - 2);
+            if (h->nccl_mode) {
+                Owner& R = h->owners[0];
+                CUDA_TRY(h, cudaSetDevice(R.dev));
+                const bool root = (ok == h->rank);
+                if (root) CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_panel[k], 0));
+                if (!root && k >= 2) {
+                    tqr_status st = wait_all_u(R, R.s_comm, k - 2);
                     if (st) return st;
-                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_look[k - 2], 0));
+                    CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
                 }
-                const PanelRefs src = own_refs(h, *O, O->lidx[k]);
-                const size_t es = h->es;
-                CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_tiles[slot], k * vt), D.dev, h->at(src.V, k * vt), O->dev,
-                                                es * (size_t)(p - k) * vt, D.s_comm));
-                CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_T[slot], k * tsz), D.dev, h->at(src.T, k * tsz), O->dev,
-                                                es * (size_t)(p - k) * tsz, D.s_comm));
-                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, src.Vexp, O->dev, es * (size_t)vt, D.s_comm));
+                if (h->profile) { CUDA_TRY(h, cudaEventRecord(R.tb0[k], R.s_comm)); }
+                PanelRefs b = root ? own_refs(h, R, R.lidx[k]) : recv_refs(h, R, slot);
+                const ncclDataType_t dt = h->f32() ? ncclFloat32 : ncclFloat64;
+                void* bv = h->at(b.V, k * vt);
+                void* bt = h->at(b.T, k * tsz);
+                NCCL_TRY(h, h->nccl->GroupStart());
+                NCCL_TRY(h, h->nccl->Broadcast(bv, bv, (size_t)(p - k) * vt, dt, ok, h->comm, R.s_comm));
+                NCCL_TRY(h, h->nccl->Broadcast(bt, bt, (size_t)(p - k) * tsz, dt, ok, h->comm, R.s_comm));
+                NCCL_TRY(h, h->nccl->Broadcast(b.Vexp, b.Vexp, (size_t)vt, dt, ok, h->comm, R.s_comm));
                 if (h->ndom(k) > 1) {
-                    const size_t nd = h->ndom(k);
-                    CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_M[slot], D.dev, src.M, O->dev, es * nd * vt, D.s_comm));
-                    CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_MT[slot], D.dev, src.MT, O->dev, es * nd * tsz, D.s_comm));
+                    const size_t D = h->ndom(k);
+                    NCCL_TRY(h, h->nccl->Broadcast(b.M, b.M, D * vt, dt, ok, h->comm, R.s_comm));
+                    NCCL_TRY(h, h->nccl->Broadcast(b.MT, b.MT, D * tsz, dt, ok, h->comm, R.s_comm));
                 }
-                CUDA_TRY(h, cudaEventRecord(D.ev_recv[k], D.s_comm));
+                NCCL_TRY(h, h->nccl->GroupEnd());
+                CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
+                if (h->profile) {
+                    CUDA_TRY(h, cudaEventRecord(R.tb1[k], R.s_comm));
+                    R.tb_used[k] = 1;
+                    h->stats[3].flops += (double)es * ((p - k) * (vt + tsz) + vt);
+                }
+            } else if (h->ipc_mode) {
+                // root: copy into every receiver's IPC-mapped slot k%2 once that receiver has freed
+                // it (its step k-2 updates are done), then raise the receiver's READY flag.
+                // receiver: free the slot at the root, wait for READY.  All waits are on local flags.
+                Owner& R = h->owners[0];
+                CUDA_TRY(h, cudaSetDevice(R.dev));
+                const uint64_t val = (uint64_t)epoch0 + 1 + k;
+                if (ok == h->rank) {
+                    CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_panel[k], 0));
+                    if (h->profile) CUDA_TRY(h, cudaEventRecord(R.tb0[k], R.s_comm));
+                    const PanelRefs src = own_refs(h, R, R.lidx[k]);
+                    std::vector<int> order;   // the lookahead owner (column k+1) first
+                    if (k + 1 < q && h->owner_of[k + 1] != h->rank) order.push_back(h->owner_of[k + 1]);
+                    for (int d = 0; d < h->world; ++d)
+                        if (d != h->rank && (order.empty() || d != order[0])) order.push_back(d);
+                    for (int d : order) {
+                        if (!needs(d, k)) continue;
+                        IpcPeer& P = h->peers[d];
+                        CUDA_TRY(h, tqr::sig_wait_geq(R.s_comm, h->flags64 + F_FREED + 2 * d + slot, val));
+                        CUDA_TRY(h, cudaMemcpyAsync(h->at(P.rb[slot][0], k * vt), h->at(src.V, k * vt),
+                                                    es * (size_t)(p - k) * vt, cudaMemcpyDefault, R.s_comm));
+                        CUDA_TRY(h, cudaMemcpyAsync(h->at(P.rb[slot][1], k * tsz), h->at(src.T, k * tsz),
+                                                    es * (size_t)(p - k) * tsz, cudaMemcpyDefault, R.s_comm));
+                        CUDA_TRY(h, cudaMemcpyAsync(P.rb[slot][2], src.Vexp, es * (size_t)vt, cudaMemcpyDefault, R.s_comm));
+                        if (h->ndom(k) > 1) {
+                            const size_t nd = h->ndom(k);
+                            CUDA_TRY(h, cudaMemcpyAsync(P.rb[slot][3], src.M, es * nd * vt, cudaMemcpyDefault, R.s_comm));
+                            CUDA_TRY(h, cudaMemcpyAsync(P.rb[slot][4], src.MT, es * nd * tsz, cudaMemcpyDefault, R.s_comm));
+                        }
+                        CUDA_TRY(h, tqr::sig_write(R.s_comm, P.flags + F_READY + slot, val));
+                        if (h->profile) h->stats[3].flops += (double)es * ((p - k) * (vt + tsz) + vt);
+                    }
+                    if (h->profile) { CUDA_TRY(h, cudaEventRecord(R.tb1[k], R.s_comm)); R.tb_used[k] = 1; }
+                } else if (needs(h->rank, k)) {
+                    if (k >= 2) {
+                        tqr_status st = wait_all_u(R, R.s_comm, k - 2);
+                        if (st) return st;
+                        CUDA_TRY(h, cudaStreamWaitEvent(R.s_comm, R.ev_look[k - 2], 0));
+                    }
+                    CUDA_TRY(h, tqr::sig_write(R.s_comm, h->peers[ok].flags + F_FREED + 2 * h->rank + slot, val));
+                    CUDA_TRY(h, tqr::sig_wait_geq(R.s_comm, h->flags64 + F_READY + slot, val));
+                    CUDA_TRY(h, cudaEventRecord(R.ev_recv[k], R.s_comm));
+                }
+            } else {
+                for (auto& D : h->owners) {
+                    if (D.id == ok || !needs(D.id, k)) continue;
+                    CUDA_TRY(h, cudaSetDevice(D.dev));
+                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_panel[k], 0));
+                    if (k >= 2) {
+                        tqr_status st = wait_all_u(D, D.s_comm, k - 2);
+                        if (st) return st;
+                        CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, D.ev_look[k - 2], 0));
+                    }
+                    if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tb0[k], D.s_comm));
+                    const PanelRefs src = own_refs(h, *O, O->lidx[k]);
+                    CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_tiles[slot], k * vt), D.dev, h->at(src.V, k * vt), O->dev,
+                                                    es * (size_t)(p - k) * vt, D.s_comm));
+                    CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_T[slot], k * tsz), D.dev, h->at(src.T, k * tsz), O->dev,
+                                                    es * (size_t)(p - k) * tsz, D.s_comm));
+                    CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, src.Vexp, O->dev, es * (size_t)vt, D.s_comm));
+                    if (h->ndom(k) > 1) {
+                        const size_t nd = h->ndom(k);
+                        CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_M[slot], D.dev, src.M, O->dev, es * nd * vt, D.s_comm));
+                        CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_MT[slot], D.dev, src.MT, O->dev, es * nd * tsz, D.s_comm));
+                    }
+                    CUDA_TRY(h, cudaEventRecord(D.ev_recv[k], D.s_comm));
+                    if (h->profile) {
+                        CUDA_TRY(h, cudaEventRecord(D.tb1[k], D.s_comm));
+                        D.tb_used[k] = 1;
+                        h->stats[3].flops += (double)es * ((p - k) * (vt + tsz) + vt);
+                    }
+                }
             }
+            emit(1, k, k, k, ok);
+            continue;
         }
-        // ---- UPDATE(k) on every local owner
+        // ---- UPDATE(k): the run of UPDATE records of step k (one per column j > k of a local owner)
+        size_t end = pos;
+        int64_t nsched = 0;
+        while (end < nrec && sched[5 * end] == 2 && sched[5 * end + 1] == k) { ++end; ++nsched; }
+        pos = end;
+        int64_t nlocal = 0;
         for (auto& D : h->owners) {
             CUDA_TRY(h, cudaSetDevice(D.dev));
             const bool mine = (D.id == ok);
@@ -1226,6 +1570,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
             // local columns j > k form a suffix [first, ncols) of D.cols
             int first = (int)(std::upper_bound(D.cols.begin(), D.cols.end(), k) - D.cols.begin());
             const int nloc = (int)D.cols.size();
+            nlocal += nloc - first;
             const bool la = h->lookahead && first < nloc && D.cols[first] == k + 1;
             if (la) {
                 // lookahead: column k+1 first, on a high-priority stream.  FP64 flat panel of this
@@ -1241,6 +1586,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 const int wl = w_look(h);
                 CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, sl,
                                    &h->launches, ovl ? D.flags : nullptr, epoch0 + (unsigned)k + 1));
+                emit(2, k, k, D.cols[first], ok);
                 if (ovl) {   // PANEL(k+1) (panel stream) after the lookahead
                     CUDA_TRY(h, cudaEventRecord(D.ev_look[k], sl));
                     CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_look[k], 0));
@@ -1274,12 +1620,9 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                         // for its last one covers them all; one launch keeps the chunk's columns
                         // concurrent (per-column launches on one stream would run one at a time)
                         CUDA_TRY(h, cudaStreamWaitEvent(su, D.ev_load[g0 + (ng - 1) * gs], 0));
-                        CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, gs, k, wb, ng * (nb / wb), true, su,
-                                           &h->launches));
-                    } else {
-                        CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, gs, k, wb, ng * (nb / wb), true, su,
-                                           &h->launches));
                     }
+                    CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, g0, gs, k, wb, ng * (nb / wb), true, su,
+                                       &h->launches));
                     if (h->profile) {
                         CUDA_TRY(h, cudaEventRecord(D.tm1[uu][k], su));
                         D.tm_used[uu][k] = 1;
@@ -1287,16 +1630,20 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                         h->stats[0].count += 1;
                     }
                 }
+                for (int c = 0; c < ng; ++c) emit(2, k, k, D.cols[g0 + c * gs], ok);
                 CUDA_TRY(h, cudaEventRecord(D.ev_u[uu][k], su));
             }
         }
+        if (nlocal != nsched)
+            return fail(h, TQR_ERR_STATE, "schedule: step %d lists %lld updates, %lld local columns", k,
+                        (long long)nsched, (long long)nlocal);
     }
     tqr_status st = sync_all(h);
     if (st) return st;
     if (h->profile) {
         for (auto& o : h->owners) {
             CUDA_TRY(h, cudaSetDevice(o.dev));
-            std::vector<std::pair<double, double>> iv, ip;
+            std::vector<std::pair<double, double>> iv, ip, ib_;
             for (int k = 0; k < q; ++k) {
                 float a = 0.f, b = 0.f;
                 for (int uu = 0; uu < S; ++uu)
@@ -1312,10 +1659,32 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                     h->stats[1].count += 1;
                     h->stats[1].flops += flops_panel(h, k);
                 }
+                if (o.tb_used[k] && o.dev == h->owners[0].dev) {
+                    CUDA_TRY(h, cudaEventElapsedTime(&a, o.tref[0], o.tb0[k]));
+                    CUDA_TRY(h, cudaEventElapsedTime(&b, o.tref[0], o.tb1[k]));
+                    ib_.push_back({a, b});
+                    h->stats[3].count += 1;
+                }
             }
             h->stats[0].ms += union_ms(iv);
             h->stats[1].ms += union_ms(ip);
+            h->stats[3].ms += union_ms(ib_);
         }
+    }
+    if (h->ipc_mode) {
+        // next factorization: my receive slots 0 / 1 are free for its steps 0 / 1 (at every root);
+        // this factorization is complete on this rank (apply/solve replication may read it)
+        Owner& R = h->owners[0];
+        CUDA_TRY(h, cudaSetDevice(R.dev));
+        h->fact_id = (uint64_t)epoch0 + 1;
+        for (int d = 0; d < h->world; ++d) {
+            if (d == h->rank) continue;
+            for (int sl = 0; sl < 2; ++sl)
+                CUDA_TRY(h, tqr::sig_write(R.s_comm, h->peers[d].flags + F_FREED + 2 * h->rank + sl,
+                                           (uint64_t)h->epoch + 1 + sl));
+            CUDA_TRY(h, tqr::sig_write(R.s_comm, h->peers[d].flags + F_DONE + h->rank, h->fact_id));
+        }
+        CUDA_TRY(h, cudaStreamSynchronize(R.s_comm));
     }
     h->factored = true;
     return TQR_OK;
@@ -1335,6 +1704,7 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
         if (o.cols.empty()) continue;
         CUDA_TRY(h, cudaSetDevice(o.dev));
         const int nc = (int)o.cols.size();
+        if (h->profile) CUDA_TRY(h, cudaEventRecord(o.tl[2], o.s_upd));
         if (pi.kind == Mem::Device && pi.dev == o.dev) {
             CUDA_TRY(h, from_tiles(h, A, lda, nb * lda, o.tiles, o.cols_dev, nc, h->m, h->n, 0, o.s_upd));
             h->launches++;
@@ -1350,8 +1720,11 @@ tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
                                               group_cols(h, j), cudaMemcpyDefault, o.s_upd));
             }
         }
+        if (h->profile) CUDA_TRY(h, cudaEventRecord(o.tl[3], o.s_upd));
     }
-    return sync_all(h);
+    tqr_status st = sync_all(h);
+    if (st) return st;
+    return layout_stat(h, 2);
 }
 
 // Streamed factor of a single tile column in tree mode (C4-like, one owner, one CTA per domain):
@@ -1427,6 +1800,7 @@ tqr_status factor_streamed_tall(tqr_plan h, void* A, int64_t lda) {
     st = sync_all(h);
     if (st) return st;
     h->factored = true;
+    h->fact_gen += 1;
     return TQR_OK;
 }
 }  // namespace
@@ -1489,12 +1863,155 @@ tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
 }
 
 // ------------------------------------------------------------------ apply Q^T / Q, solve
-static tqr_status single_device(tqr_plan h, int* dev) {
-    if (h->multiproc()) return fail(h, TQR_ERR_UNSUPPORTED, "apply/solve: multi-process plans not supported in this build");
-    *dev = h->owners[0].dev;
+// Owners on several GPUs, or several processes: apply/solve run on a single-owner replica of the
+// factorization on this process's device, gathered once per factorization (peer copies / IPC
+// pulls from the owners' memory / ncclBroadcast from each column's owner).
+static bool needs_replica(tqr_plan h) {
+    if (h->multiproc()) return true;
+    if (const char* e = getenv("TQR_FORCE_REPLICA")) if (atoi(e) != 0 && h->owners.size() > 1) return true;
     for (auto& o : h->owners)
-        if (o.dev != *dev) return fail(h, TQR_ERR_UNSUPPORTED, "apply/solve: owners on several GPUs not supported in this build");
+        if (o.dev != h->owners[0].dev) return true;
+    return false;
+}
+
+static tqr_status ensure_replica(tqr_plan h) {
+    if (h->rep && h->rep_gen == h->fact_gen) return TQR_OK;
+    const int dev = h->owners[0].dev;
+    CUDA_TRY(h, cudaSetDevice(dev));
+    if (!h->rep) {
+        tqr_options o{};
+        o.logical_devices = 1;
+        o.no_lookahead = 1;
+        o.row_split = -1;
+        o.tree_domain = h->tree_L > 0 ? h->tree_L : -1;
+        o.tree_group = h->tree_G > 1 ? h->tree_G : -1;
+        tqr_status st = tqr_create_ex(h->m, h->n, h->nb, h->ib, h->dtype, 1, nullptr, 0, &o, &h->rep);
+        if (st) return fail(h, st, "apply/solve replica: %s", g_create_error.c_str());
+        if (h->rep->tree_L != h->tree_L || h->rep->tree_G != h->tree_G || h->rep->dmax != h->dmax)
+            return fail(h, TQR_ERR_STATE, "apply/solve replica: elimination tree mismatch");
+    }
+    tqr_plan r = h->rep;
+    Owner& RO = r->owners[0];                       // owns every column, lidx[j] == j
+    const int64_t p = h->p, tile = (int64_t)h->nb * h->nb, tsz = (int64_t)h->ib * h->nb, vt = h->vt;
+    const int64_t dm = h->tree_L > 0 ? h->dmax : 0;
+    const int64_t sz[6] = {p * tile, p * vt, p * tsz, vt, dm * vt, dm * tsz};   // per column, elements
+    void* dst_base[6] = {RO.tiles, RO.Vimg, RO.T, RO.Vexp, RO.Mimg, RO.MT};
+    cudaStream_t s = RO.s_upd;
+    const size_t es = h->es;
+    if (h->nccl_mode) NCCL_TRY(h, h->nccl->GroupStart());
+    for (int j = 0; j < h->q; ++j) {
+        const int o = h->owner_of[j];
+        int lc = 0;                                 // j's index among its owner's columns
+        for (int jj = 0; jj < j; ++jj) lc += (h->owner_of[jj] == o);
+        const bool local = !h->multiproc() || o == h->rank;
+        Owner* O = local ? h->local(o) : nullptr;
+        void* src_base[6] = {nullptr};
+        int src_dev = dev;
+        if (local) {
+            void* b[6] = {O->tiles, O->Vimg, O->T, O->Vexp, O->Mimg, O->MT};
+            for (int f = 0; f < 6; ++f) src_base[f] = b[f];
+            src_dev = O->dev;
+        } else if (h->ipc_mode) {
+            for (int f = 0; f < 6; ++f) src_base[f] = h->peers[o].st[f];
+            src_dev = h->peers[o].dev;
+            CUDA_TRY(h, tqr::sig_wait_geq(s, h->flags64 + F_DONE + o, h->fact_id));
+        }
+        for (int f = 0; f < 6; ++f) {
+            if (sz[f] == 0) continue;
+            void* dst = h->at(dst_base[f], (int64_t)j * sz[f]);
+            if (h->nccl_mode) {
+                const void* sb = local ? h->at(src_base[f], (int64_t)lc * sz[f]) : dst;
+                NCCL_TRY(h, h->nccl->Broadcast(sb, dst, (size_t)sz[f], h->f32() ? ncclFloat32 : ncclFloat64, o, h->comm, s));
+            } else {
+                CUDA_TRY(h, cudaMemcpyPeerAsync(dst, dev, h->at(src_base[f], (int64_t)lc * sz[f]), src_dev, es * sz[f], s));
+            }
+        }
+    }
+    if (h->nccl_mode) NCCL_TRY(h, h->nccl->GroupEnd());
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    r->factored = true;
+    h->rep_gen = h->fact_gen;
     return TQR_OK;
+}
+
+// IPC collective epilogue of apply / solve: return only when every rank has finished reading the
+// owners' storage (so no rank's next factor overwrites reflectors a peer is still pulling).
+static tqr_status ipc_apply_barrier(tqr_plan h) {
+    if (!h->ipc_mode) return TQR_OK;
+    h->apply_seq += 1;
+    cudaStream_t s = h->owners[0].s_comm;
+    CUDA_TRY(h, cudaSetDevice(h->owners[0].dev));
+    for (int d = 0; d < h->world; ++d)
+        if (d != h->rank) CUDA_TRY(h, tqr::sig_write(s, h->peers[d].flags + F_APPLIED + h->rank, h->apply_seq));
+    for (int d = 0; d < h->world; ++d)
+        if (d != h->rank) CUDA_TRY(h, tqr::sig_wait_geq(s, h->flags64 + F_APPLIED + d, h->apply_seq));
+    CUDA_TRY(h, cudaStreamSynchronize(s));
+    return TQR_OK;
+}
+
+static tqr_status single_device(tqr_plan h, int* dev) {
+    *dev = h->owners[0].dev;
+    return TQR_OK;
+}
+
+// Row split (single process): Q = diag(Q_g) E Q_top, where E embeds the stacked first nb rows of
+// every owner's block (the rows of R_g) into the stage-2 stack.  Q^T B: every block B_g <- Q_g^T B_g,
+// gather the blocks' first nb rows into the stack, stack <- Q_top^T stack, scatter back.  Q B: the
+// reverse.  Stack rows past an owner's block (rows_g < nb) are zero rows of the stacked R and stay
+// zero under Q_top, so they are dropped.  solve_ls: the stack is solved by the stage-2 plan (its R is
+// the final R) and X comes from the stack's first n rows.
+static tqr_status rs_apply(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs, bool solve) {
+    if (h->multiproc()) return fail(h, TQR_ERR_UNSUPPORTED, "apply/solve: multi-process row-split plans keep Q distributed");
+    const bool fwd = solve || trans == 'T' || trans == 't';
+    const int G = h->ndev, nb = h->nb;
+    const int64_t es = h->es, ls = (int64_t)G * nb;
+    CUDA_TRY(h, cudaSetDevice(h->top_dev));
+    if ((size_t)(ls * nrhs) > h->bw_elems) {
+        if (h->bw) cudaFree(h->bw);
+        h->bw = nullptr;
+        h->bw_elems = 0;
+        CUDA_TRY(h, cudaMalloc(&h->bw, (size_t)(ls * nrhs) * es));
+        h->bw_elems = (size_t)(ls * nrhs);
+    }
+    auto kids_apply = [&](char tr) -> tqr_status {
+        for (size_t i = 0; i < h->kids.size(); ++i) {
+            CUDA_TRY(h, cudaSetDevice(h->kid_dev[i]));
+            const int g = h->kid_owner[i];
+            tqr_status st = tqr_apply_qt(h->kids[i], tr, static_cast<char*>(B) + h->rs_r0[g] * es, ldb, nrhs);
+            if (st) return kid_fail(h, h->kids[i], st);
+        }
+        return TQR_OK;
+    };
+    auto gather = [&](bool in) -> tqr_status {
+        CUDA_TRY(h, cudaSetDevice(h->top_dev));
+        if (in) CUDA_TRY(h, cudaMemset(h->bw, 0, (size_t)(ls * nrhs) * es));
+        for (int g = 0; g < G; ++g) {
+            const int64_t rows = std::min<int64_t>(nb, h->rs_rows[g]);
+            char* Bg = static_cast<char*>(B) + h->rs_r0[g] * es;
+            char* Sg = static_cast<char*>(h->bw) + (int64_t)g * nb * es;
+            if (in) CUDA_TRY(h, cudaMemcpy2D(Sg, ls * es, Bg, ldb * es, rows * es, nrhs, cudaMemcpyDefault));
+            else CUDA_TRY(h, cudaMemcpy2D(Bg, ldb * es, Sg, ls * es, rows * es, nrhs, cudaMemcpyDefault));
+        }
+        return TQR_OK;
+    };
+    tqr_status st = TQR_OK;
+    if (fwd) {
+        if ((st = kids_apply('T')) || (st = gather(true))) return st;
+        CUDA_TRY(h, cudaSetDevice(h->top_dev));
+        st = solve ? tqr_solve_ls(h->top, h->bw, ls, nrhs) : tqr_apply_qt(h->top, 'T', h->bw, ls, nrhs);
+        if (st) return kid_fail(h, h->top, st);
+        if (solve) {
+            CUDA_TRY(h, cudaMemcpy2D(B, ldb * es, h->bw, ls * es, h->n * es, nrhs, cudaMemcpyDefault));
+            return TQR_OK;
+        }
+        return gather(false);
+    }
+    if ((st = gather(true))) return st;
+    CUDA_TRY(h, cudaSetDevice(h->top_dev));
+    st = tqr_apply_qt(h->top, 'N', h->bw, ls, nrhs);
+    if (st) return kid_fail(h, h->top, st);
+    if ((st = gather(false))) return st;
+    return kids_apply('N');
 }
 
 // Bw (mp x 32*nslices, ld ldw) <- Q^T Bw (forward over the panels) or Q Bw (reverse).
@@ -1560,9 +2077,18 @@ tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nr
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "apply_qt before a successful factor");
     if (!(trans == 'T' || trans == 't' || trans == 'N' || trans == 'n')) return fail(h, TQR_ERR_ARG, "trans must be 'T' or 'N'");
-    if (h->rs) return fail(h, TQR_ERR_UNSUPPORTED, "apply_qt: row-split plans keep Q distributed (not supported)");
     if (nrhs < 0 || (nrhs > 0 && (!B || ldb < h->m))) return fail(h, TQR_ERR_ARG, "apply_qt: bad B/ldb/nrhs");
     if (nrhs == 0) return TQR_OK;
+    if (h->rs) return rs_apply(h, trans, B, ldb, nrhs, false);
+    if (needs_replica(h)) {
+        tqr_status st = ensure_replica(h);
+        if (!st) {
+            st = tqr_apply_qt(h->rep, trans, B, ldb, nrhs);
+            if (st) st = fail(h, st, "apply_qt (replica): %s", tqr_last_error(h->rep));
+        }
+        tqr_status sb = ipc_apply_barrier(h);
+        return st ? st : sb;
+    }
     int dev = 0;
     tqr_status st = single_device(h, &dev);
     if (st) return st;
@@ -1587,8 +2113,17 @@ tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "solve_ls before a successful factor");
     if (nrhs < 0 || (nrhs > 0 && (!B || ldb < h->m))) return fail(h, TQR_ERR_ARG, "solve_ls: bad B/ldb/nrhs");
-    if (h->rs) return fail(h, TQR_ERR_UNSUPPORTED, "solve_ls: row-split plans keep Q distributed (not supported)");
     if (nrhs == 0) return TQR_OK;
+    if (h->rs) return rs_apply(h, 'T', B, ldb, nrhs, true);
+    if (needs_replica(h)) {
+        tqr_status st = ensure_replica(h);
+        if (!st) {
+            st = tqr_solve_ls(h->rep, B, ldb, nrhs);
+            if (st) st = fail(h, st, "solve_ls (replica): %s", tqr_last_error(h->rep));
+        }
+        tqr_status sb = ipc_apply_barrier(h);
+        return st ? st : sb;
+    }
     int dev = 0;
     tqr_status st = single_device(h, &dev);
     if (st) return st;

@@ -116,6 +116,13 @@ cudaError_t launch_widen(const float* src, double* dst, int64_t n, cudaStream_t 
 cudaError_t launch_narrow_panel(int nb, int ib, const double* sc, const double* T64, float* tiles, float* T32,
                                 float* Vimg, float* Vexp, int k, int p, cudaStream_t s);
 int64_t f32_img_tile(int nb, int ib);
+
+// ---- stream-ordered 64-bit flags of the CUDA-IPC transport (tqr_signal.cu)
+// *addr = v after all prior work of s (addr may be peer / IPC-mapped memory)
+cudaError_t sig_write(cudaStream_t s, uint64_t* addr, uint64_t v);
+// later work of s waits until (int64_t)(*addr - v) >= 0 (addr: this process's device memory)
+cudaError_t sig_wait_geq(cudaStream_t s, const uint64_t* addr, uint64_t v);
+bool signal_uses_memops();
 size_t panel_smem_bytes(int nb, int ib);
 size_t update_smem_bytes(int nb, int ib, int w);
 

@@ -57,12 +57,15 @@ def _worker(rank, world, guide, m, n, nb, ib, seed, port, out_dir):
                 tiles[(k, k)] = np.where(np.triu(np.ones((nb, nb), bool)), r, tiles[(k, k)])
                 tiles[(i, k)], Tf[(i, k)] = b, t
         elif op == tqr.OP_BCAST:
-            # payload: reflector tiles k..p-1 of column k and their T factors
-            size = (p - k) * nb * nb + (p - k) * ib * nb
+            # payload, as the executor sends it: the reflector images of tiles k..p-1
+            # of column k, their T factors, and the explicit unit-lower V of the diagonal tile
+            # (Vexp: the UNMQR operand; the diagonal tile itself holds R above its diagonal)
+            size = (p - k) * nb * nb + (p - k) * ib * nb + nb * nb
             buf = torch.zeros(size, dtype=torch.float64)
             if root == rank:
+                vexp = np.tril(tiles[(k, k)], -1) + np.eye(nb)
                 parts = [tiles[(i, k)].ravel(order="F") for i in range(k, p)] + \
-                        [Tf[(i, k)].ravel(order="F") for i in range(k, p)]
+                        [Tf[(i, k)].ravel(order="F") for i in range(k, p)] + [vexp.ravel(order="F")]
                 buf.copy_(torch.from_numpy(np.concatenate(parts)))
             dist.broadcast(buf, src=root)
             bytes_seen.append(8 * size)
@@ -71,11 +74,14 @@ def _worker(rank, world, guide, m, n, nb, ib, seed, port, out_dir):
             off = (p - k) * nb * nb
             Tt = [v[off + (i - k) * ib * nb: off + (i - k + 1) * ib * nb].reshape((ib, nb), order="F")
                   for i in range(k, p)]
-            panels[k] = (Vt, Tt)
+            off += (p - k) * ib * nb
+            Vexp = v[off:off + nb * nb].reshape((nb, nb), order="F")
+            assert np.all(np.triu(Vexp, 1) == 0) and np.all(np.diag(Vexp) == 1.0)
+            panels[k] = (Vt, Tt, Vexp)
         elif op == tqr.OP_UPDATE:
             assert guide[j % len(guide)] == rank and j > k
-            Vt, Tt = panels[k]
-            c, info = lap.dgemqrt(Vt[0], Tt[0], tiles[(k, j)], side="L", trans="T")
+            Vt, Tt, Vexp = panels[k]
+            c, info = lap.dgemqrt(np.asfortranarray(Vexp), Tt[0], tiles[(k, j)], side="L", trans="T")
             assert info == 0
             tiles[(k, j)] = c
             for i in range(k + 1, p):
@@ -110,7 +116,8 @@ def test_distributed_schedule_and_broadcast(tmp_path, world, guide):
     ref = oracle.qr(synthetic.gaussian(m, n, seed)).R
     assert colnorm_rel_err(R, ref) <= 1e-10
     p = m // nb
-    assert list(np.load(tmp_path / "bytes.npy")) == [8 * ((m - k * nb) * nb + (p - k) * ib * nb) for k in range(n // nb)]
+    assert list(np.load(tmp_path / "bytes.npy")) == [8 * ((m - k * nb) * nb + (p - k) * ib * nb + nb * nb)
+                                                     for k in range(n // nb)]
 
 
 def _rowsplit_worker(rank, world, m, n, nb, ib, seed, port, out_dir):

@@ -55,6 +55,13 @@ def thin_q_and_residual(plan, A, Rfull):
     return Q, np.linalg.norm(A - QR) / np.linalg.norm(A)
 
 
+def lapack_orth(A):
+    """||Q^T Q - I||_F of LAPACK's Householder QR (numpy.linalg.qr) on the same input: the
+    context printed next to a failing orthogonality check (reading Q19)."""
+    Ql, _ = np.linalg.qr(A)
+    return float(np.linalg.norm(Ql.T @ Ql - np.eye(A.shape[1])))
+
+
 GRIDS = [
     # (m, n, nb, ib)  -- tile grids p x q
     (64, 64, 64, 16),       # 1x1: GEQRT only
@@ -82,7 +89,7 @@ def test_factor_matches_oracle(m, n, nb, ib):
     Q, res = thin_q_and_residual(plan, A, Rg)
     assert res <= RES_TOL, res
     orth = np.linalg.norm(Q.T @ Q - np.eye(n))
-    assert orth <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0)), orth
+    assert orth <= ORTH_TOL, (orth, lapack_orth(A))
     plan.close()
 
 
@@ -108,7 +115,8 @@ def test_ragged_matches_oracle(m, n, nb, ib):
     assert np.all(np.tril(Rg, -1) == 0.0)
     Q, res = thin_q_and_residual(plan, A, Rg)
     assert res <= RES_TOL, res
-    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0))
+    orth = np.linalg.norm(Q.T @ Q - np.eye(n))
+    assert orth <= ORTH_TOL, (orth, lapack_orth(A))
     B = synthetic.gaussian(m, 3, 3000 + m)
     Bd = dev_colmajor(B)
     plan.solve_ls(Bd)
@@ -272,8 +280,60 @@ def test_logical_devices_partition_bitwise(ndev, guide):
     _, R1 = gpu_qr(A, nb, ib)
     plan, Rp = gpu_qr(A, nb, ib, ndev=ndev, guide=guide, logical_devices=True)
     assert np.array_equal(np.triu(Rp[:n]), np.triu(R1[:n]))
+    assert colnorm_rel_err(np.triu(Rp[:n]), oracle.qr(A).R) <= R_TOL          # and against the oracle
+    Q, res = thin_q_and_residual(plan, A, Rp)                                  # multi-owner apply
+    assert res <= RES_TOL and np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL
     g = guide if guide is not None else list(range(ndev))
     assert [plan.owner(j) for j in range(n // nb)] == [g[j % len(g)] for j in range(n // nb)]
+    # the executor consumed the DAG schedule: per step, PANEL + BCAST + every owner's UPDATE columns
+    sched = sorted({r for d in range(ndev) for r in tqr.tqr_schedule(m, n, nb, ndev, guide, d)}, key=lambda r: (r[1], r[0], r[3]))
+    assert sorted(plan.issued_ops(), key=lambda r: (r[1], r[0], r[3])) == sched
+
+
+@pytest.mark.parametrize("ndev,guide,tree", [(3, [1, 0, 1, 0, 1, 2], -1), (2, [1, 0], 2)])
+def test_replica_apply_bitwise(ndev, guide, tree, monkeypatch):
+    """apply/solve on a multi-GPU or multi-process plan run on a single-owner replica gathered from
+    the owners (TQR_FORCE_REPLICA exercises that path with logical owners on one GPU): bitwise the
+    in-place multi-owner apply, and against the oracle."""
+    m, n, nb, ib = 768, 512, 64, 16
+    A = synthetic.gaussian(m, n, 8200 + ndev)
+    B = synthetic.gaussian(m, 5, 8300)
+    plan, Rg = gpu_qr(A, nb, ib, ndev=ndev, guide=guide, logical_devices=True, tree_domain=tree)
+    out = {}
+    for mode in ("direct", "replica"):
+        if mode == "replica":
+            monkeypatch.setenv("TQR_FORCE_REPLICA", "1")
+        Bd = dev_colmajor(B)
+        plan.apply_qt(Bd, "T")
+        QtB = to_np(Bd)
+        plan.apply_qt(Bd, "N")
+        Xd = dev_colmajor(B)
+        plan.solve_ls(Xd)
+        out[mode] = (QtB, to_np(Bd), to_np(Xd))
+    for a, b in zip(out["direct"], out["replica"]):
+        assert np.array_equal(a, b)
+    np.testing.assert_allclose(out["replica"][2][:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
+    plan.close()
+
+
+@pytest.mark.parametrize("scale", [1e300, 1e200, 1e-200, 1e-300])
+@pytest.mark.parametrize("m,n,nb,ib,kw", [(256, 256, 64, 16, {}), (1024, 512, 512, 32, {}),
+                                          (4096, 512, 512, 32, {"tree_domain": 2})])
+def test_extreme_scaling_matches_oracle(scale, m, n, nb, ib, kw):
+    """dlarfg/dnrm2 semantics (reading Q26): entries ~1e+-200 / 1e+-300 overflow or underflow a
+    plain sum of squares; factor_block redoes such a column on an exactly power-of-two scaled x.
+    R(cA) = c R(A): compare with the (scaled-norm) oracle and LAPACK, and Q stays orthogonal."""
+    A = synthetic.gaussian(m, n, 6100 + m + n) * scale
+    plan, Rg = gpu_qr(A, nb, ib, **kw)
+    R = np.triu(Rg[:n])
+    assert np.all(np.isfinite(R))
+    assert colnorm_rel_err(R, oracle.qr(A).R) <= R_TOL
+    assert colnorm_rel_err(R, np.linalg.qr(A, mode="r")) <= R_TOL
+    Q, _ = thin_q_and_residual(plan, A, Rg)
+    # residual on the unscaled magnitudes (numpy's norm is an unscaled sum of squares)
+    res = np.linalg.norm(A / scale - Q @ (R / scale)) / np.linalg.norm(A / scale)
+    assert res <= RES_TOL and np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL, res
+    plan.close()
 
 
 def test_lookahead_off_bitwise_identical():
@@ -391,9 +451,7 @@ def test_nccl_transport_single_rank_bitwise():
     Ad = dev_colmajor(A)
     plan.factor(Ad)
     assert np.array_equal(to_np(Ad), R1)
-    with pytest.raises(tqr.TqrError) as e:      # apply/solve are single-process only this round
-        plan.apply_qt(dev_colmajor(np.ones((m, 1))))
-    assert e.value.status == 7
+    assert colnorm_rel_err(np.triu(R1[:n]), oracle.qr(A).R) <= R_TOL
 
 
 @pytest.mark.parametrize("m,n,nb,ib,ndev", [
@@ -423,9 +481,16 @@ def test_row_split_matches_oracle(m, n, nb, ib, ndev):
     Rh = np.asfortranarray(np.full((m, n), 3.0))
     plan.store_r(Rh)
     assert np.array_equal(Rh, Rg)
-    with pytest.raises(tqr.TqrError) as e:
-        plan.apply_qt(dev_colmajor(np.ones((m, 1))))
-    assert e.value.status == 7
+    # Q of a row split = diag(Q_g) E Q_top (tqr.h): thin Q, residual, Q^T A and least squares
+    Q, res = thin_q_and_residual(plan, A, Rg)
+    assert res <= RES_TOL and np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL, res
+    QtA = dev_colmajor(A)
+    plan.apply_qt(QtA, "T")
+    assert colnorm_rel_err(np.triu(to_np(QtA)[:n]), ref.R) <= R_TOL
+    B = synthetic.gaussian(m, 3, 7550 + m)
+    Bd = dev_colmajor(B)
+    plan.solve_ls(Bd)
+    np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
     plan.close()
 
 
@@ -507,14 +572,12 @@ def test_full_size_c4_tall_skinny():
         plan.apply_qt(E, "N")
         I = torch.eye(n, dtype=torch.float64, device="cuda")
         orth = float((E.t() @ E - I).norm())
-    # Flat-TS (reading Q7) chains p = 2048 TS transformations through the same R rows, so its
-    # orthogonality loss grows ~ sqrt(p) eps and measures 1.8e-13 here vs 6.1e-14 for cuSOLVER's
-    # Householder geqrf on the same input (Q19): the absolute 1e-13 bar is not
-    # met at C4 by the flat tree.  Checked relative to LAPACK-style QR on the same input.
+    # north_star's absolute bar (reading Q19: met by Householder QR at C4, LAPACK 1.5e-14 at
+    # 262144 x 512); cuSOLVER's geqrf on the same input is printed for context
     Q2, _ = torch.linalg.qr(Ad)
     orth_ref = float((Q2.t() @ Q2 - I).norm())
     print("C4 ||Q^TQ - I||_F = %.3e (cuSOLVER geqrf %.3e)" % (orth, orth_ref))
-    assert orth <= 4.0 * orth_ref and orth <= 2.5e-13
+    assert orth <= ORTH_TOL, (orth, orth_ref)
     del Ad, Rd, E, Q2
     torch.cuda.empty_cache()
 
@@ -543,7 +606,8 @@ def test_tree_matches_oracle(m, n, nb, ib, L, one_cta, monkeypatch):
     assert np.all(np.tril(Rg, -1) == 0.0)
     Q, res = thin_q_and_residual(plan, A, Rg)
     assert res <= RES_TOL, res
-    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0))
+    orth = np.linalg.norm(Q.T @ Q - np.eye(n))
+    assert orth <= ORTH_TOL, (orth, lapack_orth(A))
     B = synthetic.gaussian(m, 2, 5100 + m)
     Bd = dev_colmajor(B)
     plan.solve_ls(Bd)
@@ -570,7 +634,8 @@ def test_two_level_merge_matches_oracle(m, n, nb, ib, L, G):
     assert np.all(np.tril(Rg, -1) == 0.0)
     Q, res = thin_q_and_residual(plan, A, Rg)
     assert res <= RES_TOL, res
-    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= ORTH_TOL * max(1.0, np.sqrt(n / 256.0))
+    orth = np.linalg.norm(Q.T @ Q - np.eye(n))
+    assert orth <= ORTH_TOL, (orth, lapack_orth(A))
     B = synthetic.gaussian(m, 2, 5400 + m)
     Bd = dev_colmajor(B)
     plan.solve_ls(Bd)
@@ -583,6 +648,7 @@ def test_two_level_merge_matches_oracle(m, n, nb, ib, L, G):
     if n > nb:
         _, Rp = gpu_qr(A, nb, ib, tree_domain=L, tree_group=G, ndev=2, guide=[1, 0], logical_devices=True)
         assert np.array_equal(Rg, Rp)
+        assert colnorm_rel_err(np.triu(Rp[:n]), ref.R) <= R_TOL
 
 
 def test_tree_auto_for_single_column_and_partition():
@@ -597,5 +663,8 @@ def test_tree_auto_for_single_column_and_partition():
     m2, n2 = 1024, 512
     A2 = synthetic.gaussian(m2, n2, 5201)
     _, R1 = gpu_qr(A2, 64, 16, tree_domain=3)
-    _, R2 = gpu_qr(A2, 64, 16, tree_domain=3, ndev=3, guide=[2, 0, 1], logical_devices=True)
+    plan2, R2 = gpu_qr(A2, 64, 16, tree_domain=3, ndev=3, guide=[2, 0, 1], logical_devices=True)
     assert np.array_equal(R1, R2)
+    assert colnorm_rel_err(np.triu(R2[:n2]), oracle.qr(A2).R) <= R_TOL
+    Q, res = thin_q_and_residual(plan2, A2, R2)
+    assert res <= RES_TOL and np.linalg.norm(Q.T @ Q - np.eye(n2)) <= ORTH_TOL
