@@ -682,11 +682,13 @@ extern "C" int tqr_probe_phases(unsigned long long* out, int reset) {
     cudaMemcpyFromSymbol(out, tqr::g_phase, sizeof(unsigned long long) * 16);
     cudaMemcpyFromSymbol(out + 16, tqr::g_pphase, sizeof(unsigned long long) * 8);
     cudaMemcpyFromSymbol(out + 24, tqr::g_fphase, sizeof(unsigned long long) * 4);
+    cudaMemcpyFromSymbol(out + 28, tqr::g_cphase, sizeof(unsigned long long) * 8);
     if (reset) {
         unsigned long long z[16] = {0};
         cudaMemcpyToSymbol(tqr::g_phase, z, sizeof(z));
         cudaMemcpyToSymbol(tqr::g_pphase, z, sizeof(unsigned long long) * 8);
         cudaMemcpyToSymbol(tqr::g_fphase, z, sizeof(unsigned long long) * 4);
+        cudaMemcpyToSymbol(tqr::g_cphase, z, sizeof(unsigned long long) * 8);
     }
     return (int)cudaGetLastError();
 }

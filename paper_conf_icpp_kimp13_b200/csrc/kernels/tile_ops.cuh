@@ -32,7 +32,15 @@ __device__ unsigned long long g_fphase[4];
 #define TQR_FP(i) do { if (threadIdx.x == 0 && blockIdx.x == gridDim.x - 1) { long long _c = clock64(); \
     atomicAdd(&g_fphase[i], (unsigned long long)(_c - _fp)); _fp = _c; } } while (0)
 #define TQR_FP0() long long _fp = clock64()
+// column-step phases of factor_block (thread 0 of the last CTA): g_cphase[0] shuffle + scale,
+// [1] dots + record, [2] barrier, [3] sums + sqrt/div, [4] w_j, [5] update + store
+__device__ unsigned long long g_cphase[8];
+#define TQR_FC(i) do { if (threadIdx.x == 0 && blockIdx.x == gridDim.x - 1) { long long _c = clock64(); \
+    atomicAdd(&g_cphase[i], (unsigned long long)(_c - _fc)); _fc = _c; } } while (0)
+#define TQR_FC0() long long _fc = clock64()
 #else
+#define TQR_FC(i) do {} while (0)
+#define TQR_FC0() do {} while (0)
 #define TQR_FP(i) do {} while (0)
 #define TQR_FP0() do {} while (0)
 #define TQR_PH(i) do {} while (0)
@@ -409,10 +417,17 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
     // unscaled dots x^T a_j of every column j of the block and (GEQRT) the row-d entries a_dj;
     // after the barrier every thread forms beta, tau, scale = 1/(x0 - beta) and
     // w_j = a_dj (GEQRT) or R(c, j) (TSQRT) + scale * sum_w (x^T a_j)_w itself (v = scale x).
-    constexpr int FBW = 2 * IB + 2;          // per-warp record: dots[IB], diag row[IB], ||x||^2, exponent
-    double* fb = sm.red;                      // [2][kWarps][FBW] (double-buffered by column parity)
+    // Column record, double-buffered by column parity (fb + (c & 1) * RECN), laid out for the reads
+    // after the barrier: dots[j][w] (warp partials of x^T a_j, warp index fastest, row stride 10 so
+    // the writers' banks differ and each thread reads its columns' 8 partials as four double2), then
+    // ||x_w||^2[w], e_w[w] (or, fast path at c = 0, the block max) and the GEQRT diagonal row a_dj
+    // (written once, by the warp that owns row d).
+    constexpr int DLD = 10;                   // dots row stride (doubles)
+    constexpr int OSS = IB * DLD, OEX = OSS + kWarps, ODG = OEX + kWarps;
+    constexpr int RECN = ODG + IB + 2;        // + pad: every buffer starts 16-byte aligned
+    static_assert(RECN % 2 == 0 && 2 * RECN <= Smem<NB, IB, IB, true>::REDN, "factor record buffer");
+    double* fb = sm.red;
     double* Rout = sm.topsm;                  // TSQRT: R rows written as they are finished
-    static_assert(2 * kWarps * FBW <= Smem<NB, IB, IB, true>::REDN, "factor record buffer");
     static_assert(IB * IB <= IB * G::LDW, "Rout buffer");
     TQR_FP0();
     // Scaled norms and dots (dlarfg / dnrm2 semantics, reading Q26) at no extra barrier: each warp
@@ -422,6 +437,14 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
     // overflow (scaled |x| < 2) and nothing that matters can underflow (a term is lost only when it
     // is below 2^-1022 relative to the column's largest entry).  Powers of two are exact, so in the
     // normal range every quantity is bitwise the unscaled formula's.
+    auto sum8 = [](const double* p8, const double* f) {   // ((p0 f0 + p1 f1) + ...) as a tree
+        const double2 a0 = *reinterpret_cast<const double2*>(p8), a1 = *reinterpret_cast<const double2*>(p8 + 2);
+        const double2 a2 = *reinterpret_cast<const double2*>(p8 + 4), a3 = *reinterpret_cast<const double2*>(p8 + 6);
+        if (f == nullptr)
+            return ((a0.x + a0.y) + (a1.x + a1.y)) + ((a2.x + a2.y) + (a3.x + a3.y));
+        return ((a0.x * f[0] + a0.y * f[1]) + (a1.x * f[2] + a1.y * f[3])) +
+               ((a2.x * f[4] + a2.y * f[5]) + (a3.x * f[6] + a3.y * f[7]));
+    };
 
 #pragma unroll
     for (int mfc = 0; mfc < G::MF; ++mfc) {
@@ -429,7 +452,8 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
         for (int gc = 0; gc < 8; ++gc) {
             const int c = mfc * 8 + gc;
             const int d = dbase + c;
-            double* fbp = fb + (c & 1) * (kWarps * FBW);
+            double* fbp = fb + (c & 1) * RECN;
+            TQR_FC0();
             // 1. x = column c on my rows (from the lane holding it, same t), masked to rows > d (GEQRT),
             //    scaled by 2^-ew (ew = exponent of the warp's largest |x|)
             double xv[G::NF][2];
@@ -457,81 +481,95 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                     xv[nf][1] *= sw;
                 }
             }
-            double ss = 0.0;
+            TQR_FC(0);
+            // ||x_w||^2 and the dots x_w^T a_j of the columns of groups >= mfc, two accumulators each
+            double ss0 = 0.0, ss1 = 0.0;
             if (g == 0) {
 #pragma unroll
-                for (int nf = 0; nf < G::NF; ++nf) ss += xv[nf][0] * xv[nf][0] + xv[nf][1] * xv[nf][1];
+                for (int nf = 0; nf < G::NF; ++nf) {
+                    ss0 += xv[nf][0] * xv[nf][0];
+                    ss1 += xv[nf][1] * xv[nf][1];
+                }
             }
-            // column groups mf < mfc hold columns j < c only (finished): no dots, no update
-            double pd[G::MF], p0[G::MF];
+            double ss = ss0 + ss1;
+            // GEQRT: the warp owning row d publishes the diagonal row a_dj (j = mf*8 + g) once
+            const bool own_d = GE && (d / G::RW) == wq;
+            const int td = ((d % G::RW) % 8) >> 1, ed = d & 1;
+            double pd[G::MF];
 #pragma unroll
             for (int mf = mfc; mf < G::MF; ++mf) {
-                double sdot = 0.0, sdiag = 0.0;
+                double s0 = 0.0, s1 = 0.0, sdiag = 0.0;
 #pragma unroll
-                for (int nf = 0; nf < G::NF; ++nf)
-#pragma unroll
-                    for (int e = 0; e < 2; ++e) {
-                        sdot += xv[nf][e] * X.acc[mf][nf][e];
-                        if (GE && rbase + nf * 8 + e == d) sdiag = X.acc[mf][nf][e];
+                for (int nf = 0; nf < G::NF; ++nf) {
+                    s0 += xv[nf][0] * X.acc[mf][nf][0];
+                    s1 += xv[nf][1] * X.acc[mf][nf][1];
+                    if (GE) {
+                        if (rbase + nf * 8 == d) sdiag = X.acc[mf][nf][0];
+                        if (rbase + nf * 8 + 1 == d) sdiag = X.acc[mf][nf][1];
                     }
+                }
+                double sdot = s0 + s1;
                 sdot += __shfl_xor_sync(0xffffffffu, sdot, 1);
                 sdot += __shfl_xor_sync(0xffffffffu, sdot, 2);
                 pd[mf] = sdot;
                 if (GE) {
-                    sdiag += __shfl_xor_sync(0xffffffffu, sdiag, 1);
-                    sdiag += __shfl_xor_sync(0xffffffffu, sdiag, 2);
+                    sdiag = __shfl_sync(0xffffffffu, sdiag, g * 4 + td);
+                    if (own_d && t == 0) fbp[ODG + mf * 8 + g] = sdiag;
                 }
-                p0[mf] = sdiag;
             }
+            (void)ed;
             ss += __shfl_xor_sync(0xffffffffu, ss, 1);
             ss += __shfl_xor_sync(0xffffffffu, ss, 2);
             if (t == 0) {
-                double* rec = fbp + wq * FBW;
 #pragma unroll
-                for (int mf = mfc; mf < G::MF; ++mf) {
-                    rec[mf * 8 + g] = pd[mf];
-                    if (GE) rec[IB + mf * 8 + g] = p0[mf];
-                }
+                for (int mf = mfc; mf < G::MF; ++mf) fbp[(mf * 8 + g) * DLD + wq] = pd[mf];
                 if (g == 0) {
-                    rec[2 * IB] = ss;
-                    if (SCALED) rec[2 * IB + 1] = (double)ew;
-                    else if (c == 0) rec[2 * IB + 1] = wmax;
+                    fbp[OSS + wq] = ss;
+                    if (SCALED) fbp[OEX + wq] = (double)ew;
+                    else if (c == 0) fbp[OEX + wq] = wmax;
                 }
             }
+            TQR_FC(1);
             __syncthreads();
+            TQR_FC(2);
             // 2. reflector (dlarfg convention, readings Q1/Q4): beta = -sgn(x0) ||(x0, x)||, in units
             //    of 2^ec; fw[w] = 2^(e_w - ec) brings warp w's partials to that scale
-            double x0 = 0.0, xn2 = 0.0, fw[kWarps];
+            // the dots of my columns first (independent of the reflector: overlaps sqrt / div)
+            double fw[kWarps];
             int ec = 0;
+            const double x0 = GE ? fbp[ODG + c] : sm.Rsm[c * IB + c];
             if constexpr (SCALED) {
                 int ewv[kWarps];
                 ec = kNoExp;
 #pragma unroll
                 for (int w = 0; w < kWarps; ++w) {
-                    ewv[w] = (int)fbp[w * FBW + 2 * IB + 1];
+                    ewv[w] = (int)fbp[OEX + w];
                     ec = max(ec, ewv[w]);
-                    if (GE) x0 += fbp[w * FBW + IB + c];
                 }
-                if (!GE) x0 = sm.Rsm[c * IB + c];
                 ec = max(ec, exp2_floor(x0));
                 if (ec == kNoExp) ec = 0;                                 // x == 0 and x0 == 0
 #pragma unroll
-                for (int w = 0; w < kWarps; ++w) {
-                    fw[w] = pow2s(ewv[w] - ec);
-                    xn2 += fbp[w * FBW + 2 * IB] * (fw[w] * fw[w]);
-                }
-            } else {
+                for (int w = 0; w < kWarps; ++w) fw[w] = pow2s(ewv[w] - ec);
+            }
+            double dsum[G::MF], basev[G::MF];
 #pragma unroll
-                for (int w = 0; w < kWarps; ++w) {
-                    fw[w] = 1.0;
-                    xn2 += fbp[w * FBW + 2 * IB];
-                    if (GE) x0 += fbp[w * FBW + IB + c];
-                }
-                if (!GE) x0 = sm.Rsm[c * IB + c];
+            for (int mf = mfc; mf < G::MF; ++mf) {
+                const int j = mf * 8 + g;
+                dsum[mf] = sum8(fbp + j * DLD, SCALED ? fw : nullptr);
+                basev[mf] = GE ? fbp[ODG + j] : sm.Rsm[c * IB + j];
+            }
+            double xn2;
+            if constexpr (SCALED) {
+                double f2[kWarps];
+#pragma unroll
+                for (int w = 0; w < kWarps; ++w) f2[w] = fw[w] * fw[w];
+                xn2 = sum8(fbp + OSS, f2);
+            } else {
+                xn2 = sum8(fbp + OSS, nullptr);
                 if (c == 0) {
                     double bm = 0.0;
 #pragma unroll
-                    for (int w = 0; w < kWarps; ++w) bm = fmax(bm, fbp[w * FBW + 2 * IB + 1]);
+                    for (int w = 0; w < kWarps; ++w) bm = fmax(bm, fbp[OEX + w]);
                     bad = bad || !(bm <= 0x1p490);
                 }
                 // GEQRT's last tile column has no sub-column (legitimately x = 0, tau = 0)
@@ -553,6 +591,7 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
 #pragma unroll
                 for (int w = 0; w < kWarps; ++w) vfac = (w == wq) ? scale * fw[w] : vfac;
             }
+            TQR_FC(3);
             // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = x / (x0 - beta) (+ e_d)
             double tw[G::MF];
 #pragma unroll
@@ -560,18 +599,12 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 const int j = mf * 8 + g;
                 tw[mf] = 0.0;
                 if (j > c) {
-                    double dsum = 0.0, base = 0.0;
-#pragma unroll
-                    for (int w = 0; w < kWarps; ++w) {
-                        dsum += fbp[w * FBW + j] * fw[w];
-                        if (GE) base += fbp[w * FBW + IB + j];
-                    }
-                    if (!GE) base = sm.Rsm[c * IB + j];
-                    const double wj = base + scale * dsum;
+                    const double wj = basev[mf] + scale * dsum[mf];
                     tw[mf] = tau * wj;
-                    if (!GE && wq == 0 && t == 0) Rout[c * IB + j] = base - tau * wj;
+                    if (!GE && wq == 0 && t == 0) Rout[c * IB + j] = basev[mf] - tau * wj;
                 }
             }
+            TQR_FC(4);
 #pragma unroll
             for (int mf = mfc; mf < G::MF; ++mf) {
 #pragma unroll
@@ -597,6 +630,7 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 sm.tau[c] = tau;
                 if (!GE) Rout[c * IB + c] = beta;
             }
+            TQR_FC(5);
         }
     }
     if (!SCALED && bad) {                   // CTA-uniform: sm.Rsm untouched, the caller redoes the block

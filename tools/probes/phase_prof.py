@@ -14,7 +14,7 @@ m, n, nb, ib, seed = CONFIGS[cfg]
 g = torch.Generator(device="cuda").manual_seed(seed)
 A = torch.randn((n, m), dtype=torch.float64, device="cuda", generator=g).t()
 R = torch.empty((n, m), dtype=torch.float64, device="cuda").t()
-buf = (ctypes.c_ulonglong * 28)()
+buf = (ctypes.c_ulonglong * 36)()
 with tqr.Plan(m, n, nb, ib) as p:
     p.load(A); p.factor_tiles(); p.store_r(R)
     L.tqr_probe_phases(buf, 1)
@@ -39,3 +39,8 @@ ft = sum(buf[24 + i] for i in range(3))
 if ft:
     print("factor_block (last CTA): columns %.1f Mcyc, Gram %.1f Mcyc, dlarft recurrence %.1f Mcyc" %
           tuple(buf[24 + i] / 1e6 for i in range(3)))
+ct = sum(buf[28 + i] for i in range(6))
+if ct:
+    print("factor_block column step (last CTA):", ", ".join("%s %.1f%%" % (nm, 100.0 * buf[28 + i] / ct) for i, nm in
+          enumerate(["shuffle+scale", "dots+record", "barrier", "sums+sqrt/div", "w_j", "update+store"])),
+          "total Mcycles %.1f" % (ct / 1e6))
