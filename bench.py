@@ -135,15 +135,15 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def oracle_sample(cfg_name, nthreads=0):
-    """Bounded CPU-oracle sample of the config: Algorithm 1 on the first min(n, 2048) columns
-    of the config's own matrix (same generator, same rows; ~10 s of host work for C5).
+def oracle_sample(cfg_name, nthreads=0, ncols=None):
+    """Bounded CPU-oracle sample of the config: Algorithm 1 on the first min(n, 2048) (or ncols)
+    columns of the config's own matrix (same generator, same rows; ~10 s of host work for C5).
     Returns (GFLOP/s, seconds, desc)."""
     import numpy as np
     import oracle
     import synthetic
     m, n, nb, ib, seed = CONFIGS[cfg_name]
-    ns = min(n, SAMPLE_COLS)
+    ns = min(n, SAMPLE_COLS if ncols is None else ncols)
     rows = np.arange(m, dtype=np.uint64)
     A = np.empty((m, ns), order="F")
     for j in range(ns):
@@ -151,7 +151,8 @@ def oracle_sample(cfg_name, nthreads=0):
     t0 = time.perf_counter()
     oracle.qr(A, nthreads=nthreads)
     dt = time.perf_counter() - t0
-    return flops(m, ns) / dt / 1e9, dt, "oracle.qr on A[:, :%d] of %s (%dx%d), %.2f s" % (ns, cfg_name, m, ns, dt)
+    return flops(m, ns) / dt / 1e9, dt, "oracle.qr on A[:, :%d] of %s (%dx%d), %s, %.2f s" % (
+        ns, cfg_name, m, ns, "1 thread" if nthreads == 1 else "all host cores", dt)
 
 
 def run_reference(args):
@@ -385,6 +386,9 @@ def main():
         v, dt, desc = oracle_sample(args.config)
         cpu = {"value": round(v, 3), "unit": "GFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
                "sample": desc}
+        # the oracle on one thread as well (a narrower sample: ~1-3 s of host work)
+        v1, dt1, desc1 = oracle_sample(args.config, nthreads=1, ncols=min(256, CONFIGS[args.config][1]))
+        cpu["single_thread"] = {"value": round(v1, 3), "unit": "GFLOP/s", "cores": 1, "sample": desc1}
 
     if rank == 0:
         # achieved = algorithmic flops of all bulk-update launches / their device-busy time

@@ -235,20 +235,32 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
     }
     TQR_PH(0);
 
-    // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib), one pass per half
+    // ---- (1) GEMM1: partial W^T(col, ib) = sum_{my rows} X(row, col) V(row, ib), one pass per half.
+    //      Narrow slices (MF <= 2: the lookahead and panel sub-slices) have only MF * JC accumulator
+    //      chains per half; they get a second set for odd row fragments (NP = 2) so consecutive
+    //      DMMAs do not wait on each other's results, summed once at the end.
+#ifdef TQR_GEMM1_SPLIT
+    constexpr int NP = (G::MF <= 2) ? 2 : 1;
+#else
+    constexpr int NP = 1;
+#endif
     double c1[2][G::MF][G::JC][2];
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
         mbar_wait(&sm.mbar[wq][h], (vph >> h) & 1u);
         vph ^= 1u << h;
         const double* vh = &sm.Vst[wq][h][0][0];
+        double cp[NP][G::MF][G::JC][2];
 #pragma unroll
-        for (int mf = 0; mf < G::MF; ++mf)
+        for (int pp = 0; pp < NP; ++pp)
 #pragma unroll
-            for (int j = 0; j < G::JC; ++j) c1[h][mf][j][0] = c1[h][mf][j][1] = 0.0;
+            for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+                for (int j = 0; j < G::JC; ++j) cp[pp][mf][j][0] = cp[pp][mf][j][1] = 0.0;
 #pragma unroll
         for (int nf = 0; nf < G::NF; ++nf) {
             if (KM && (rbase + nf * 8 + 8 <= kmin || rbase + nf * 8 >= kmax)) continue;  // V rows all zero (warp-uniform)
+            const int pp = (NP == 2) ? (nf & 1) : 0;
             double2 b[G::JC];
 #pragma unroll
             for (int j = 0; j < G::JC; ++j)
@@ -256,12 +268,23 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
 #pragma unroll
             for (int mf = 0; mf < G::MF; ++mf)
 #pragma unroll
-                for (int j = 0; j < G::JC; ++j) dmma(c1[h][mf][j][0], c1[h][mf][j][1], X.acc[mf][nf][0], b[j].x);
+                for (int j = 0; j < G::JC; ++j) dmma(cp[pp][mf][j][0], cp[pp][mf][j][1], X.acc[mf][nf][0], b[j].x);
 #pragma unroll
             for (int mf = 0; mf < G::MF; ++mf)
 #pragma unroll
-                for (int j = 0; j < G::JC; ++j) dmma(c1[h][mf][j][0], c1[h][mf][j][1], X.acc[mf][nf][1], b[j].y);
+                for (int j = 0; j < G::JC; ++j) dmma(cp[pp][mf][j][0], cp[pp][mf][j][1], X.acc[mf][nf][1], b[j].y);
         }
+#pragma unroll
+        for (int mf = 0; mf < G::MF; ++mf)
+#pragma unroll
+            for (int j = 0; j < G::JC; ++j) {
+                c1[h][mf][j][0] = cp[0][mf][j][0];
+                c1[h][mf][j][1] = cp[0][mf][j][1];
+                if (NP == 2) {
+                    c1[h][mf][j][0] += cp[NP - 1][mf][j][0];
+                    c1[h][mf][j][1] += cp[NP - 1][mf][j][1];
+                }
+            }
         TQR_PH(1 + h);
     }
     // c1[h][mf][j] = W^T[col mf*8+g][ib h*HC + j*8 + 2t + e]
@@ -437,7 +460,10 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
     // overflow (scaled |x| < 2) and nothing that matters can underflow (a term is lost only when it
     // is below 2^-1022 relative to the column's largest entry).  Powers of two are exact, so in the
     // normal range every quantity is bitwise the unscaled formula's.
-    auto sum8 = [](const double* p8, const double* f) {   // ((p0 f0 + p1 f1) + ...) as a tree
+    // Sum of the 8 warp partials at p8 (times fw[w] = 2^(e_w - ec) when scaled), as a tree:
+    // ((p0 + p1) + (p2 + p3)) + ((p4 + p5) + (p6 + p7)); four 16-byte loads.  (Splitting the loads
+    // across a lane quad + two butterflies measured slower: profiles/r02_factor_phases.txt.)
+    auto sum8 = [](const double* p8, const double* f) {
         const double2 a0 = *reinterpret_cast<const double2*>(p8), a1 = *reinterpret_cast<const double2*>(p8 + 2);
         const double2 a2 = *reinterpret_cast<const double2*>(p8 + 4), a3 = *reinterpret_cast<const double2*>(p8 + 6);
         if (f == nullptr)
@@ -536,6 +562,7 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
             //    of 2^ec; fw[w] = 2^(e_w - ec) brings warp w's partials to that scale
             // the dots of my columns first (independent of the reflector: overlaps sqrt / div)
             double fw[kWarps];
+            double fwq = 1.0;
             int ec = 0;
             const double x0 = GE ? fbp[ODG + c] : sm.Rsm[c * IB + c];
             if constexpr (SCALED) {
@@ -550,6 +577,7 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 if (ec == kNoExp) ec = 0;                                 // x == 0 and x0 == 0
 #pragma unroll
                 for (int w = 0; w < kWarps; ++w) fw[w] = pow2s(ewv[w] - ec);
+                fwq = pow2s(ew - ec);
             }
             double dsum[G::MF], basev[G::MF];
 #pragma unroll
@@ -586,11 +614,7 @@ __device__ __forceinline__ bool factor_block(Slice<NB, IB, IB>& X, Smem<NB, IB, 
                 beta = SCALED ? bs * pow2s(ec / 2) * pow2s(ec - ec / 2) : bs;   // back to the caller's scale
             }
             // v on my rows = (x 2^-ew) 2^(ew - ec) scale (+ e_d); |v| <= 1
-            double vfac = scale;
-            if constexpr (SCALED) {
-#pragma unroll
-                for (int w = 0; w < kWarps; ++w) vfac = (w == wq) ? scale * fw[w] : vfac;
-            }
+            const double vfac = SCALED ? scale * fwq : scale;
             TQR_FC(3);
             // 3. w_j for my columns j > c, then X(:, j) -= tau v w_j with v = x / (x0 - beta) (+ e_d)
             double tw[G::MF];

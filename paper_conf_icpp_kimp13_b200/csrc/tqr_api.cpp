@@ -25,9 +25,14 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <chrono>
+#include <new>
+#include <thread>
 #include <numeric>
 #include <string>
 #include <vector>
+
+#include <nvtx3/nvToolsExt.h>
 
 #include "nccl_dl.h"
 #include "tqr_internal.h"
@@ -38,6 +43,19 @@ using tqr::UpdateArgs;
 namespace {
 
 thread_local std::string g_create_error;
+
+// NVTX ranges (header-only NVTX v3: free when no profiler is attached) around the ABI phases and
+// every factorization step, so an nsys / ncu timeline shows load, PANEL(k) / BCAST(k) / UPDATE(k),
+// R out, apply and solve.
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    NvtxRange(const char* fmt, int k) {
+        char b[48];
+        snprintf(b, sizeof(b), fmt, k);
+        nvtxRangePushA(b);
+    }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 struct Owner {
     int id = 0;
@@ -150,6 +168,7 @@ struct tqr_plan_s {
     void* prog = nullptr;           // wavefront apply progress flags (q * nslices)
     size_t prog_n = 0;
     bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
+    bool la_fits = true;            // ... only when its spinning CTAs leave SMs for the whole panel grid
     bool streamed = false;
     bool domains_done = false;      // streamed tall factor: the TS domains were launched per row chunk
     bool cp_probe = false;          // TQR_CRITICAL_PATH_PROBE=1 (diagnostic, wrong results): skip the
@@ -295,14 +314,18 @@ void build_schedule(int64_t q, const std::vector<int32_t>& owner_of, int rank, s
     }
 }
 
+constexpr int64_t kMaxGuide = 1 << 20;   // longest distribution guide array accepted
+
+// Returns an empty vector when the guide would exceed kMaxGuide entries.
 std::vector<int32_t> generate_guide(const std::vector<int32_t>& rates) {
     // GET_RATIO: divide by the gcd; GENERATE_ARRAY: argmax + decrement,
     // lowest ID on ties (readings Q11/Q12).
     int g = 0;
     for (int r : rates) g = std::gcd(g, r);
     std::vector<int32_t> ratio(rates.size());
-    int sum = 0;
+    int64_t sum = 0;   // 64-bit: sum of up to ndev ratios of up to 2^31
     for (size_t i = 0; i < rates.size(); ++i) { ratio[i] = rates[i] / g; sum += ratio[i]; }
+    if (sum > kMaxGuide) return {};
     std::vector<int32_t> ga(sum);
     for (int i = 0; i < sum; ++i) {
         int best = 0;
@@ -352,15 +375,56 @@ tqr_status ensure_io(tqr_plan h, Owner& o) {
 // valid (unpadded) columns of column group j
 int64_t group_cols(const tqr_plan_s* h, int64_t j) { return std::min<int64_t>(h->nb, h->n - j * h->nb); }
 
+// Wait for a stream.  Multi-process plans poll instead of blocking, so a peer that died (its flags
+// never raised, its NCCL kernels never matched) turns into an error after TQR_PEER_TIMEOUT_S
+// seconds (default 600) instead of a hang; NCCL's asynchronous error is checked while polling and
+// the communicator aborted on failure.  The plan is poisoned either way.
+tqr_status wait_stream(tqr_plan h, cudaStream_t st) {
+    if (!h->multiproc()) {
+        CUDA_TRY(h, cudaStreamSynchronize(st));
+        return TQR_OK;
+    }
+    static const double limit = [] {
+        const char* e = getenv("TQR_PEER_TIMEOUT_S");
+        return e ? atof(e) : 600.0;
+    }();
+    const auto t0 = std::chrono::steady_clock::now();
+    for (int it = 0;; ++it) {
+        const cudaError_t q = cudaStreamQuery(st);
+        if (q == cudaSuccess) return TQR_OK;
+        if (q != cudaErrorNotReady)
+            return fail(h, TQR_ERR_CUDA, "stream wait: %s", cudaGetErrorString(q));
+        if (h->nccl_mode && h->comm && h->nccl && h->nccl->CommGetAsyncError) {
+            ncclResult_t ar = ncclSuccess;
+            if (h->nccl->CommGetAsyncError(h->comm, &ar) == ncclSuccess && ar != ncclSuccess && ar != ncclInProgress) {
+                if (h->nccl->CommAbort) h->nccl->CommAbort(h->comm);
+                h->comm = nullptr;
+                return fail(h, TQR_ERR_NCCL, "NCCL asynchronous error: %s", h->nccl->GetErrorString(ar));
+            }
+        }
+        const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+        if (el > limit) {
+            if (h->nccl_mode && h->comm && h->nccl && h->nccl->CommAbort) {
+                h->nccl->CommAbort(h->comm);
+                h->comm = nullptr;
+            }
+            return fail(h, h->nccl_mode ? TQR_ERR_NCCL : TQR_ERR_CUDA,
+                        "no progress from a peer rank for %.0f s (TQR_PEER_TIMEOUT_S)", el);
+        }
+        std::this_thread::sleep_for(std::chrono::microseconds(it < 1000 ? 20 : 200));
+    }
+}
+
 tqr_status sync_all(tqr_plan h) {
     for (auto& o : h->owners) {
         CUDA_TRY(h, cudaSetDevice(o.dev));
-        CUDA_TRY(h, cudaStreamSynchronize(o.s_panel));
-        CUDA_TRY(h, cudaStreamSynchronize(o.s_upd));
-        CUDA_TRY(h, cudaStreamSynchronize(o.s_comm));
-        for (auto su : o.s_u) CUDA_TRY(h, cudaStreamSynchronize(su));
-        if (o.s_io) CUDA_TRY(h, cudaStreamSynchronize(o.s_io));
-        if (o.s_look) CUDA_TRY(h, cudaStreamSynchronize(o.s_look));
+        std::vector<cudaStream_t> ss = {o.s_panel, o.s_upd, o.s_comm, o.s_io, o.s_look};
+        ss.insert(ss.end(), o.s_u.begin(), o.s_u.end());
+        for (auto st : ss) {
+            if (!st) continue;
+            tqr_status r = wait_stream(h, st);
+            if (r) return r;
+        }
     }
     return TQR_OK;
 }
@@ -386,11 +450,12 @@ const char* tqr_status_string(tqr_status s) {
 
 const char* tqr_last_error(tqr_plan h) { return h ? h->err.c_str() : g_create_error.c_str(); }
 
-tqr_status tqr_generate_guide(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len) {
+static tqr_status tqr_generate_guide_impl(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len) {
     if (!rates || ndev < 1 || !len) return fail(nullptr, TQR_ERR_ARG, "generate_guide: bad arguments");
     std::vector<int32_t> r(rates, rates + ndev);
     for (int x : r) if (x <= 0) return fail(nullptr, TQR_ERR_ARG, "generate_guide: rates must be > 0");
     auto ga = generate_guide(r);
+    if (ga.empty()) return fail(nullptr, TQR_ERR_ARG, "generate_guide: guide longer than %lld entries", (long long)kMaxGuide);
     *len = (int32_t)ga.size();
     if (guide) {
         if (cap < (int32_t)ga.size()) return fail(nullptr, TQR_ERR_ARG, "generate_guide: capacity %d < %zu", cap, ga.size());
@@ -411,7 +476,7 @@ static tqr_status validate_guide(int32_t ndev, const int32_t* guide, int32_t gui
     return TQR_OK;
 }
 
-tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const int32_t* guide, int32_t guide_len,
+static tqr_status tqr_schedule_impl(int64_t m, int64_t n, int32_t nb, int32_t ndev, const int32_t* guide, int32_t guide_len,
                         int32_t rank, int32_t* ops, int64_t cap, int64_t* count) {
     if (m < 1 || n < 1 || m < n || nb < 1 || ndev < 1 || rank < 0 || rank >= ndev || !count)
         return fail(nullptr, TQR_ERR_ARG, "schedule: bad arguments");
@@ -590,7 +655,7 @@ static tqr_status create_row_split(int64_t m, int64_t n, int32_t nb, int32_t ib,
     return TQR_OK;
 }
 
-tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
+static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
                          const int32_t* guide, int32_t guide_len, const tqr_options* opt, tqr_plan* out) {
     if (!out) return fail(nullptr, TQR_ERR_ARG, "out is NULL");
     *out = nullptr;
@@ -690,6 +755,16 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
     if (ib < 32 && h->panel_split > 2) h->panel_split = 2;
     if (const char* e = getenv("TQR_PANEL_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->panel_split = v; }
     if (ib / h->panel_split < 8) h->panel_split = 1;
+    {
+        // The overlapped lookahead's CTAs spin until the panel publishes tiles; forward progress needs
+        // the whole panel grid resident beside them (one CTA per SM each; fewer SMs under MPS / a
+        // partitioned GPU): otherwise the lookahead waits for the panel on the stream instead.
+        int sms = 148;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+        const int panel_ctas = (nb / ib) * (h->panel_split + 1);
+        const int look_ctas = nb / (nb >= 256 ? 8 : 16);
+        h->la_fits = panel_ctas + look_ctas <= sms;
+    }
     h->owner_of.resize(h->q);
     for (int j = 0; j < h->q; ++j) h->owner_of[j] = g[j % g.size()];
 
@@ -710,8 +785,11 @@ tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype
             if (h->owner_of[j] == ow.id) { ow.lidx[j] = (int32_t)ow.cols.size(); ow.cols.push_back(j); }
         if (cudaSetDevice(ow.dev) != cudaSuccess) return bail(fail(h, TQR_ERR_CUDA, "cudaSetDevice(%d)", ow.dev));
         auto mk = [&](cudaStream_t* s, int prio) { return cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, prio); };
+        // the overlapped lookahead (it spins on the panel's flags) one priority level below the panel,
+        // so freed SMs go to the panel's CTAs first (prio_hi is the numerically smallest value)
+        const int prio_look = std::min(prio_lo, prio_hi + 1);
         if (mk(&ow.s_panel, prio_hi) || mk(&ow.s_upd, prio_lo) || mk(&ow.s_comm, prio_hi) || mk(&ow.s_io, prio_hi) ||
-            mk(&ow.s_look, prio_hi))
+            mk(&ow.s_look, prio_look))
             return bail(fail(h, TQR_ERR_CUDA, "stream creation failed"));
         const int S = h->nstreams_alloc();
         ow.s_u.assign(S, nullptr);
@@ -853,7 +931,7 @@ void peer_from_ptrs(IpcPeer& pr, void* const ptr[kNH]) {
 }
 }  // namespace
 
-tqr_status tqr_ipc_handle(tqr_plan h, void* buf, int64_t cap, int64_t* len) {
+static tqr_status tqr_ipc_handle_impl(tqr_plan h, void* buf, int64_t cap, int64_t* len) {
     if (!h || !len) return fail(h, TQR_ERR_ARG, "ipc_handle: bad arguments");
     if (!h->ipc_mode) return fail(h, TQR_ERR_STATE, "ipc_handle: the plan does not use the IPC transport");
     *len = (int64_t)sizeof(IpcBlob);
@@ -877,7 +955,7 @@ tqr_status tqr_ipc_handle(tqr_plan h, void* buf, int64_t cap, int64_t* len) {
     return TQR_OK;
 }
 
-tqr_status tqr_ipc_connect(tqr_plan h, const void* all, int64_t len) {
+static tqr_status tqr_ipc_connect_impl(tqr_plan h, const void* all, int64_t len) {
     if (!h || !all) return fail(h, TQR_ERR_ARG, "ipc_connect: bad arguments");
     if (!h->ipc_mode) return fail(h, TQR_ERR_STATE, "ipc_connect: the plan does not use the IPC transport");
     if (h->ipc_connected) return fail(h, TQR_ERR_STATE, "ipc_connect: already connected");
@@ -1173,12 +1251,12 @@ tqr_status rs_factor(tqr_plan h) {
         if (h->f32()) CUDA_TRY(h, tqr::launch_zero_below_blocks<float>((float*)h->stk, ld, ld, n, nb, h->rs_stream));
         else CUDA_TRY(h, tqr::launch_zero_below_blocks<double>((double*)h->stk, ld, ld, n, nb, h->rs_stream));
         h->launches++;
-        CUDA_TRY(h, cudaStreamSynchronize(h->rs_stream));
+        { tqr_status ws = wait_stream(h, h->rs_stream); if (ws) return ws; }
         tqr_status st = tqr_load(h->top, h->stk, ld);
         if (!st) st = tqr_factor_tiles(h->top);
         if (st) return kid_fail(h, h->top, st);
     } else {
-        CUDA_TRY(h, cudaStreamSynchronize(h->rs_stream));
+        { tqr_status ws = wait_stream(h, h->rs_stream); if (ws) return ws; }
     }
     h->factored = true;
     return TQR_OK;
@@ -1229,7 +1307,8 @@ tqr_status layout_stat(tqr_plan h, int ev) {
 }
 }  // namespace
 
-tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
+static tqr_status tqr_load_impl(tqr_plan h, const void* A, int64_t lda) {
+    NvtxRange nvtx_("tqr_load (a1)");
     if (!h) return TQR_ERR_ARG;
     if (h->rs) {
         if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
@@ -1363,7 +1442,8 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
 }
 }  // namespace
 
-tqr_status tqr_factor_tiles(tqr_plan h) {
+static tqr_status tqr_factor_tiles_impl(tqr_plan h) {
+    NvtxRange nvtx_("tqr_factor_tiles (a2-a7)");
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (h->ipc_mode && !h->ipc_connected) return fail(h, TQR_ERR_STATE, "IPC plan not connected (tqr_ipc_connect)");
@@ -1414,6 +1494,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
     while (pos < nrec) {
         const int op = sched[5 * pos], k = sched[5 * pos + 1];
         const int ok = h->owner_of[k];
+        NvtxRange nvtx_op(op == 0 ? "PANEL(%d)" : (op == 1 ? "BCAST(%d)" : "UPDATE(%d)"), k);
         Owner* O = h->local(ok);
         if (op == 0) {
             // ---- PANEL(k)
@@ -1578,7 +1659,7 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                 // dispatched first) and waits per reflector tile on the panel's flags; otherwise it
                 // follows the whole panel (or the broadcast) on the panel stream.
                 // (not with logical owners: several owners' lookaheads could then spin on one GPU)
-                const bool ovl = mine && h->la_overlap && !h->logical && !h->f32() && h->ndom(k) == 1;
+                const bool ovl = mine && h->la_overlap && h->la_fits && !h->logical && !h->f32() && h->ndom(k) == 1;
                 cudaStream_t sl = ovl ? D.s_look : D.s_panel;
                 if (!ovl) CUDA_TRY(h, cudaStreamWaitEvent(sl, ready, 0));
                 if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_u[stream_of(first, (int)D.cols.size())][k - 1], 0));
@@ -1684,14 +1765,15 @@ tqr_status tqr_factor_tiles(tqr_plan h) {
                                            (uint64_t)h->epoch + 1 + sl));
             CUDA_TRY(h, tqr::sig_write(R.s_comm, h->peers[d].flags + F_DONE + h->rank, h->fact_id));
         }
-        CUDA_TRY(h, cudaStreamSynchronize(R.s_comm));
+        { tqr_status ws = wait_stream(h, R.s_comm); if (ws) return ws; }
     }
     h->factored = true;
     return TQR_OK;
 }
 
 // ------------------------------------------------------------------ a8: R out
-tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
+static tqr_status tqr_store_r_impl(tqr_plan h, void* A, int64_t lda) {
+    NvtxRange nvtx_("tqr_store_r (a8)");
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "store_r before factor");
@@ -1810,7 +1892,8 @@ tqr_status factor_streamed_tall(tqr_plan h, void* A, int64_t lda) {
 // PANEL(j) and the step-0 update of column j wait only for column j, and R of column k (a8) is
 // copied out as soon as PANEL(k) completes, so only the first column's load and the last
 // column's store are exposed.  A is in place (the columns being read are never the ones written).
-tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
+static tqr_status tqr_factor_impl(tqr_plan h, void* A, int64_t lda) {
+    NvtxRange nvtx_("tqr_factor");
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!A || lda < h->m) return fail(h, TQR_ERR_ARG, "factor: A is NULL or lda < m");
@@ -1928,7 +2011,7 @@ static tqr_status ensure_replica(tqr_plan h) {
         }
     }
     if (h->nccl_mode) NCCL_TRY(h, h->nccl->GroupEnd());
-    CUDA_TRY(h, cudaStreamSynchronize(s));
+    { tqr_status ws = wait_stream(h, s); if (ws) return ws; }
     r->factored = true;
     h->rep_gen = h->fact_gen;
     return TQR_OK;
@@ -1945,7 +2028,7 @@ static tqr_status ipc_apply_barrier(tqr_plan h) {
         if (d != h->rank) CUDA_TRY(h, tqr::sig_write(s, h->peers[d].flags + F_APPLIED + h->rank, h->apply_seq));
     for (int d = 0; d < h->world; ++d)
         if (d != h->rank) CUDA_TRY(h, tqr::sig_wait_geq(s, h->flags64 + F_APPLIED + d, h->apply_seq));
-    CUDA_TRY(h, cudaStreamSynchronize(s));
+    { tqr_status ws = wait_stream(h, s); if (ws) return ws; }
     return TQR_OK;
 }
 
@@ -2072,7 +2155,8 @@ static tqr_status stage_b(tqr_plan h, const void* B, int64_t ldb, int64_t nrhs, 
     return TQR_OK;
 }
 
-tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs) {
+static tqr_status tqr_apply_qt_impl(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs) {
+    NvtxRange nvtx_("tqr_apply_qt");
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "apply_qt before a successful factor");
@@ -2108,7 +2192,8 @@ tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nr
     return TQR_OK;
 }
 
-tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
+static tqr_status tqr_solve_ls_impl(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
+    NvtxRange nvtx_("tqr_solve_ls");
     if (!h) return TQR_ERR_ARG;
     if (h->poisoned) return fail(h, TQR_ERR_STATE, "plan poisoned by an earlier CUDA/NCCL failure");
     if (!h->factored) return fail(h, TQR_ERR_STATE, "solve_ls before a successful factor");
@@ -2170,6 +2255,109 @@ tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
     return TQR_OK;
 }
 
+// Every ABI entry point that can allocate on the host: no C++ exception crosses the boundary.
+tqr_status tqr_create_ex(int64_t m, int64_t n, int32_t nb, int32_t ib, tqr_dtype dtype, int32_t ndev,
+                         const int32_t* guide, int32_t guide_len, const tqr_options* opt, tqr_plan* out) {
+    try {
+        return tqr_create_ex_impl(m, n, nb, ib, dtype, ndev, guide, guide_len, opt, out);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_create_ex: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_create_ex: unexpected exception");
+    }
+}
+tqr_status tqr_factor(tqr_plan h, void* A, int64_t lda) {
+    try {
+        return tqr_factor_impl(h, A, lda);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_factor: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_factor: unexpected exception");
+    }
+}
+tqr_status tqr_load(tqr_plan h, const void* A, int64_t lda) {
+    try {
+        return tqr_load_impl(h, A, lda);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_load: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_load: unexpected exception");
+    }
+}
+tqr_status tqr_factor_tiles(tqr_plan h) {
+    try {
+        return tqr_factor_tiles_impl(h);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_factor_tiles: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_factor_tiles: unexpected exception");
+    }
+}
+tqr_status tqr_store_r(tqr_plan h, void* A, int64_t lda) {
+    try {
+        return tqr_store_r_impl(h, A, lda);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_store_r: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_store_r: unexpected exception");
+    }
+}
+tqr_status tqr_apply_qt(tqr_plan h, char trans, void* B, int64_t ldb, int64_t nrhs) {
+    try {
+        return tqr_apply_qt_impl(h, trans, B, ldb, nrhs);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_apply_qt: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_apply_qt: unexpected exception");
+    }
+}
+tqr_status tqr_solve_ls(tqr_plan h, void* B, int64_t ldb, int64_t nrhs) {
+    try {
+        return tqr_solve_ls_impl(h, B, ldb, nrhs);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_solve_ls: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_solve_ls: unexpected exception");
+    }
+}
+tqr_status tqr_schedule(int64_t m, int64_t n, int32_t nb, int32_t ndev, const int32_t* guide, int32_t guide_len,
+                        int32_t rank, int32_t* ops, int64_t cap, int64_t* count) {
+    try {
+        return tqr_schedule_impl(m, n, nb, ndev, guide, guide_len, rank, ops, cap, count);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_schedule: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_schedule: unexpected exception");
+    }
+}
+tqr_status tqr_generate_guide(const int32_t* rates, int32_t ndev, int32_t* guide, int32_t cap, int32_t* len) {
+    try {
+        return tqr_generate_guide_impl(rates, ndev, guide, cap, len);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_generate_guide: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_generate_guide: unexpected exception");
+    }
+}
+tqr_status tqr_ipc_connect(tqr_plan h, const void* all, int64_t len) {
+    try {
+        return tqr_ipc_connect_impl(h, all, len);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_ipc_connect: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_ipc_connect: unexpected exception");
+    }
+}
+tqr_status tqr_ipc_handle(tqr_plan h, void* buf, int64_t cap, int64_t* len) {
+    try {
+        return tqr_ipc_handle_impl(h, buf, cap, len);
+    } catch (const std::bad_alloc&) {
+        return fail(nullptr, TQR_ERR_ALLOC, "tqr_ipc_handle: host allocation failed");
+    } catch (...) {
+        return fail(nullptr, TQR_ERR_ARG, "tqr_ipc_handle: unexpected exception");
+    }
+}
+
 }  // extern "C"
 
 // ------------------------------------------------------------------ NCCL loader
@@ -2191,6 +2379,7 @@ const NcclApi* nccl_api(const char** why) {
             api.CommInitRank = (decltype(api.CommInitRank))sym("ncclCommInitRank");
             api.CommDestroy = (decltype(api.CommDestroy))sym("ncclCommDestroy");
             api.CommGetAsyncError = (decltype(api.CommGetAsyncError))sym("ncclCommGetAsyncError");
+            api.CommAbort = (decltype(api.CommAbort))sym("ncclCommAbort");
             api.Broadcast = (decltype(api.Broadcast))sym("ncclBroadcast");
             api.AllGather = (decltype(api.AllGather))sym("ncclAllGather");
             api.GroupStart = (decltype(api.GroupStart))sym("ncclGroupStart");

@@ -27,10 +27,11 @@ std::vector<int32_t> guide_for(const tqr_tile_times* t, const std::vector<int>& 
     double lo = std::numeric_limits<double>::infinity();
     for (int d : devs) lo = std::min(lo, upd_speed(t[d]));
     std::vector<int32_t> rates(devs.size());
+    // ratios clamped to [1, 4096] before the rounding cast (no int overflow for wildly mismatched rates)
     for (size_t i = 0; i < devs.size(); ++i)
-        rates[i] = std::max(1, (int)std::lround(upd_speed(t[devs[i]]) / lo));
+        rates[i] = (int32_t)std::lround(std::min(4096.0, std::max(1.0, upd_speed(t[devs[i]]) / lo)));
     int32_t len = 0;
-    tqr_generate_guide(rates.data(), (int32_t)rates.size(), nullptr, 0, &len);
+    if (tqr_generate_guide(rates.data(), (int32_t)rates.size(), nullptr, 0, &len) != TQR_OK) return {};
     std::vector<int32_t> g(len);
     tqr_generate_guide(rates.data(), (int32_t)rates.size(), g.data(), len, &len);
     return g;
@@ -84,6 +85,7 @@ tqr_status tqr_select_ndev(int32_t M, int32_t N, int32_t T, int32_t elem_size, i
     for (int p = 1; p <= ndev; ++p) {
         std::vector<int> devs(lst.begin(), lst.begin() + p);
         const std::vector<int32_t> g = guide_for(t, devs);
+        if (g.empty()) return TQR_ERR_ARG;
         // Eq. 10: trailing columns j = 1..N-1 by Eq. 12, M update tiles each
         std::vector<double> ntile(p, 0.0);
         for (int j = 1; j < N; ++j) ntile[g[j % g.size()]] += M;
