@@ -379,6 +379,19 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
             flag_wait_geq(a.wflags + (int64_t)(ti < 0 ? k : ti) * NBLK + NBLK - 1, a.wepoch);
             if (lane_id() == 0) fence_proxy_async_global();   // panel's generic stores -> bulk copies
         }
+        if (a.cflags) {                  // trailing a remote panel: tile ti's chunk landed in the slot?
+            const unsigned long long* f = a.cflags + ((ti < 0 ? k : ti) - k) / a.cchunk;
+            if (threadIdx.x == 0) {
+                for (;;) {
+                    unsigned long long x;
+                    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(x) : "l"(f) : "memory");
+                    if ((long long)(x - a.cval) >= 0) break;
+                    __nanosleep(128);
+                }
+                fence_proxy_async_global();
+            }
+            __syncthreads();
+        }
     };
     if (ntiles > 0) {
         wait_tile(tile_of(0));

@@ -93,6 +93,8 @@ struct Owner {
     std::vector<cudaEvent_t> ev_chunk, ev_dom;      // streamed tall factor: row chunk c loaded / its domains done
     std::vector<cudaStream_t> s_u;                  // bulk-update streams (column lc -> s_u[lc % S])
     std::vector<cudaEvent_t> ev_panel, ev_recv, ev_look;
+    std::vector<cudaEvent_t> ev_prepanel;           // before PANEL(k)'s launch (remote trailing lookahead)
+    unsigned long long* cflg = nullptr;             // remote trailing: chunk flags, 2 slots x kMaxChunks
     std::vector<std::vector<cudaEvent_t>> ev_u;     // ev_u[u][k]: stream u finished its step-k updates
     std::vector<std::vector<cudaEvent_t>> tm0, tm1; // profiling pairs per (u, k)
     std::vector<cudaEvent_t> tp0, tp1, tref;        // panel pairs, reference
@@ -120,6 +122,7 @@ struct IpcBlob {
     uint32_t magic;
     int32_t rank, dev, world;
     uint64_t present;            // bit i: handle i exported
+    unsigned char uuid[16];      // the GPU's UUID (ordinals differ between processes)
     cudaIpcMemHandle_t h[kNH];
 };
 constexpr uint32_t kIpcMagic = 0x54515231u;   // "TQR1"
@@ -130,10 +133,13 @@ constexpr int F_DONE = 160;      // [src]             rank src finished factoriz
 constexpr int F_APPLIED = 224;   // [src]             rank src finished apply/solve call #seq (its pulls)
 constexpr int F_RSREADY = 288;   // [src]             row split: rank src's R_g is in its rs_send (rank 0's block)
 constexpr int F_PULLED = 352;    //                   row split: rank 0 has pulled my R_g of #E (my block)
+constexpr int F_CHUNK = 384;     // [slot*64 + c]     remote trailing: chunk c of the panel in my slot (root writes)
+constexpr int kMaxChunks = 64;
 constexpr int kFlagWords = 512;
 constexpr int kIpcMaxWorld = 64;
 struct IpcPeer {
     int dev = -1;
+    unsigned char uuid[16] = {0};
     uint64_t* flags = nullptr;
     void* rb[2][5] = {{nullptr}};   // receive slot s: tiles, T, V, M, MT
     void* st[6] = {nullptr};        // tiles, Vimg, T, Vexp, Mimg, MT
@@ -169,6 +175,8 @@ struct tqr_plan_s {
     size_t prog_n = 0;
     bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
     bool la_fits = true;            // ... only when its spinning CTAs leave SMs for the whole panel grid
+    bool la_remote = false;         // the lookahead of column k+1 on ANOTHER owner trails PANEL(k) chunk by chunk
+    int la_chunk = 8;               // tiles per trailing transfer chunk
     bool streamed = false;
     bool domains_done = false;      // streamed tall factor: the TS domains were launched per row chunk
     bool cp_probe = false;          // TQR_CRITICAL_PATH_PROBE=1 (diagnostic, wrong results): skip the
@@ -288,8 +296,9 @@ void free_owner(Owner& o) {
     F(o.sc_col); F(o.sc_T); F(o.sc_Vimg); F(o.sc_Vexp); F(o.Mimg); F(o.MT); F(o.Mt);
     for (int s = 0; s < 2; ++s) { F(o.rb_M[s]); F(o.rb_MT[s]); }
     for (int s = 0; s < 2; ++s) { F(o.rb_tiles[s]); F(o.rb_T[s]); F(o.rb_V[s]); }
+    F(o.cflg);
     for (auto* v : {&o.ev_panel, &o.ev_recv, &o.ev_look, &o.tp0, &o.tp1, &o.tref, &o.ev_load, &o.ev_chunk, &o.ev_dom,
-                    &o.tb0, &o.tb1})
+                    &o.tb0, &o.tb1, &o.ev_prepanel})
         for (auto e : *v) if (e) cudaEventDestroy(e);
     for (auto e : o.tl) if (e) cudaEventDestroy(e);
     for (auto* vv : {&o.ev_u, &o.tm0, &o.tm1})
@@ -765,6 +774,18 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
         const int look_ctas = nb / (nb >= 256 ? 8 : 16);
         h->la_fits = panel_ctas + look_ctas <= sms;
     }
+    {
+        // Remote trailing lookahead: the owner of column k+1 (another owner) receives panel k in chunks
+        // of tiles as the TS chain publishes them and starts its lookahead on the first chunk.  Logical
+        // owners and IPC ranks on distinct GPUs by default (IPC ranks sharing a GPU: off, decided in
+        // tqr_ipc_connect); in-process owners on several GPUs and NCCL: opt-in / off.
+        const char* e = getenv("TQR_LA_REMOTE");
+        const int want = e ? atoi(e) : -1;
+        const bool path = h->logical || use_ipc || (want > 0 && !use_nccl);
+        h->la_remote = want != 0 && path && h->lookahead && dtype == TQR_F64 && h->tree_L == 0 && ndev > 1 &&
+                       h->la_fits;
+        h->la_chunk = std::max(8, (h->p + kMaxChunks - 1) / kMaxChunks);
+    }
     h->owner_of.resize(h->q);
     for (int j = 0; j < h->q; ++j) h->owner_of[j] = g[j % g.size()];
 
@@ -803,7 +824,7 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
             return true;
         };
         bool ok = mkev(ow.ev_panel, h->q, false) && mkev(ow.ev_recv, h->q, false) && mkev(ow.ev_look, h->q, false) &&
-                  mkev(ow.ev_load, (int)ow.cols.size(), false);
+                  mkev(ow.ev_load, (int)ow.cols.size(), false) && mkev(ow.ev_prepanel, h->q, false);
         ow.ev_u.resize(S);
         for (int u = 0; u < S && ok; ++u) ok = mkev(ow.ev_u[u], h->q, false);
         if (ok && h->profile) {
@@ -860,6 +881,11 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
             if (h->tree_L > 0 && (cudaMalloc(&ow.mflags, nfl * sizeof(unsigned)) != cudaSuccess ||
                                   cudaMemset(ow.mflags, 0, nfl * sizeof(unsigned)) != cudaSuccess))
                 return bail(fail(h, TQR_ERR_ALLOC, "flag allocation failed"));
+        }
+        if (h->la_remote && !use_ipc) {
+            if (cudaMalloc(&ow.cflg, 2 * kMaxChunks * sizeof(unsigned long long)) != cudaSuccess ||
+                cudaMemset(ow.cflg, 0, 2 * kMaxChunks * sizeof(unsigned long long)) != cudaSuccess)
+                return bail(fail(h, TQR_ERR_ALLOC, "chunk flag allocation failed"));
         }
     }
     // peer access between physical owners (single-process, several GPUs)
@@ -943,6 +969,11 @@ static tqr_status tqr_ipc_handle_impl(tqr_plan h, void* buf, int64_t cap, int64_
     b.rank = h->rank;
     b.world = h->world;
     b.dev = plan_device(h);
+    {
+        cudaDeviceProp pr;
+        CUDA_TRY(h, cudaGetDeviceProperties(&pr, b.dev));
+        std::memcpy(b.uuid, &pr.uuid, sizeof(b.uuid));
+    }
     void* ptr[kNH];
     export_ptrs(h, ptr);
     CUDA_TRY(h, cudaSetDevice(b.dev));
@@ -983,7 +1014,13 @@ static tqr_status tqr_ipc_connect_impl(tqr_plan h, const void* all, int64_t len)
         }
         peer_from_ptrs(h->peers[r], ptr);
         h->peers[r].dev = b.dev;
+        std::memcpy(h->peers[r].uuid, b.uuid, sizeof(b.uuid));
     }
+    // ranks sharing a GPU are time-sliced: a lookahead spinning on another rank's chunk flags would
+    // hold its context's slice -- no remote trailing then (same decision on every rank: all devices known)
+    for (int a = 0; a < h->world; ++a)
+        for (int b = a + 1; b < h->world; ++b)
+            if (std::memcmp(h->peers[a].uuid, h->peers[b].uuid, sizeof(h->peers[a].uuid)) == 0) h->la_remote = false;
     // arm: my receive slots 0 / 1 are free for steps 0 / 1 of the first factorization, at every
     // possible root (the flag lives in the root's block; roots only ever wait on their own block)
     cudaStream_t s = plan_comm_stream(h);
@@ -1094,7 +1131,8 @@ struct PanelRefs {
 cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const void* Vexp, void* X, int64_t col_stride,
                     int64_t tile_stride, int64_t ld, int group0, int gstride, int k_head, int p_end, int do_unmqr,
                     int w, int nslices, bool trans, cudaStream_t s, int vstride = 1,
-                    const unsigned* wflags = nullptr, unsigned wepoch = 0, int domL = 0, int njobs = 1) {
+                    const unsigned* wflags = nullptr, unsigned wepoch = 0, int domL = 0, int njobs = 1,
+                    const unsigned long long* cflags = nullptr, unsigned long long cval = 0, int cchunk = 1) {
     if (h->f32()) {
         tqr::UpdateArgsT<float> u;
         u.V = (const float*)V; u.T = (const float*)T; u.Vexp = (const float*)Vexp; u.X = (float*)X;
@@ -1107,6 +1145,7 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
     u.col_stride = col_stride; u.tile_stride = tile_stride; u.ld = ld;
     u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr; u.vstride = vstride;
     u.wflags = wflags; u.wepoch = wepoch;
+    u.cflags = cflags; u.cval = cval; u.cchunk = cchunk;
     if (domL > 0) { u.domL = domL; u.nslc = nslices; }
     return tqr::launch_update(h->nb, h->ib, w, u, nslices * njobs, trans, s);
 }
@@ -1119,12 +1158,13 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
 // reverse order.  Returns the number of launches in *nl.
 cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col_stride, int64_t tile_stride,
                    int64_t ld, int group0, int gstride, int k, int w, int nslices, bool trans, cudaStream_t s,
-                   int64_t* nl = nullptr, const unsigned* wflags = nullptr, unsigned wepoch = 0) {
+                   int64_t* nl = nullptr, const unsigned* wflags = nullptr, unsigned wepoch = 0,
+                   const unsigned long long* cflags = nullptr, unsigned long long cval = 0, int cchunk = 1) {
     const int D = h->ndom(k), L = h->tree_L;
     if (D == 1) {
         if (nl) *nl += 1;
         return update1(h, r.V, r.T, r.Vexp, X, col_stride, tile_stride, ld, group0, gstride, k, h->p, 1, w, nslices,
-                       trans, s, 1, wflags, wepoch);
+                       trans, s, 1, wflags, wepoch, 0, 1, cflags, cval, cchunk);
     }
     // all D domains in one launch (independent row ranges; job d = domain d, head k + d*L)
     auto doms = [&]() {
@@ -1503,6 +1543,8 @@ static tqr_status tqr_factor_tiles_impl(tqr_plan h) {
             CUDA_TRY(h, cudaSetDevice(O->dev));
             if (k > 0 && !h->lookahead) { tqr_status st = wait_all_u(*O, O->s_panel, k - 1); if (st) return st; }
             if (h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(O->s_panel, O->ev_load[O->lidx[k]], 0));
+            // every prerequisite of PANEL(k) done: a remote lookahead trailing it may start spinning
+            if (h->la_remote) CUDA_TRY(h, cudaEventRecord(O->ev_prepanel[k], O->s_panel));
             if (h->profile) CUDA_TRY(h, cudaEventRecord(O->tp0[k], O->s_panel));
             tqr_status st = launch_panel_step(h, *O, k, epoch0 + (unsigned)k + 1);
             if (st) return st;
@@ -1579,6 +1621,27 @@ static tqr_status tqr_factor_tiles_impl(tqr_plan h) {
                         if (!needs(d, k)) continue;
                         IpcPeer& P = h->peers[d];
                         CUDA_TRY(h, tqr::sig_wait_geq(R.s_comm, h->flags64 + F_FREED + 2 * d + slot, val));
+                        if (h->la_remote && k + 1 < q && d == h->owner_of[k + 1]) {
+                            // the lookahead owner: chunk c of tiles once PANEL(k) published its last tile
+                            // (the TS chain publishes in order), then its chunk flag; it trails the panel
+                            const int CH = h->la_chunk;
+                            for (int t0 = k, c = 0; t0 < p; t0 += CH, ++c) {
+                                const int t1 = std::min(p, t0 + CH);
+                                CUDA_TRY(h, tqr::sig_wait_geq32(R.s_comm, R.flags + (int64_t)(t1 - 1) * (nb / ib) + nb / ib - 1,
+                                                                epoch0 + (unsigned)k + 1));
+                                CUDA_TRY(h, cudaMemcpyAsync(h->at(P.rb[slot][0], t0 * vt), h->at(src.V, t0 * vt),
+                                                            es * (size_t)(t1 - t0) * vt, cudaMemcpyDefault, R.s_comm));
+                                CUDA_TRY(h, cudaMemcpyAsync(h->at(P.rb[slot][1], t0 * tsz), h->at(src.T, t0 * tsz),
+                                                            es * (size_t)(t1 - t0) * tsz, cudaMemcpyDefault, R.s_comm));
+                                if (t0 == k)
+                                    CUDA_TRY(h, cudaMemcpyAsync(P.rb[slot][2], src.Vexp, es * (size_t)vt, cudaMemcpyDefault,
+                                                                R.s_comm));
+                                CUDA_TRY(h, tqr::sig_write(R.s_comm, P.flags + F_CHUNK + slot * kMaxChunks + c, val));
+                            }
+                            CUDA_TRY(h, tqr::sig_write(R.s_comm, P.flags + F_READY + slot, val));
+                            if (h->profile) h->stats[3].flops += (double)es * ((p - k) * (vt + tsz) + vt);
+                            continue;
+                        }
                         CUDA_TRY(h, cudaMemcpyAsync(h->at(P.rb[slot][0], k * vt), h->at(src.V, k * vt),
                                                     es * (size_t)(p - k) * vt, cudaMemcpyDefault, R.s_comm));
                         CUDA_TRY(h, cudaMemcpyAsync(h->at(P.rb[slot][1], k * tsz), h->at(src.T, k * tsz),
@@ -1607,7 +1670,8 @@ static tqr_status tqr_factor_tiles_impl(tqr_plan h) {
                 for (auto& D : h->owners) {
                     if (D.id == ok || !needs(D.id, k)) continue;
                     CUDA_TRY(h, cudaSetDevice(D.dev));
-                    CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_panel[k], 0));
+                    const bool trail = h->la_remote && k + 1 < q && D.id == h->owner_of[k + 1];
+                    if (!trail) CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_panel[k], 0));
                     if (k >= 2) {
                         tqr_status st = wait_all_u(D, D.s_comm, k - 2);
                         if (st) return st;
@@ -1615,6 +1679,33 @@ static tqr_status tqr_factor_tiles_impl(tqr_plan h) {
                     }
                     if (h->profile) CUDA_TRY(h, cudaEventRecord(D.tb0[k], D.s_comm));
                     const PanelRefs src = own_refs(h, *O, O->lidx[k]);
+                    if (trail) {
+                        // the lookahead owner: chunks of tiles as PANEL(k) publishes them (stream wait on
+                        // the panel's own flags), a chunk flag after each; the lookahead trails them
+                        CUDA_TRY(h, cudaStreamWaitEvent(D.s_comm, O->ev_prepanel[k], 0));
+                        const int CH = h->la_chunk;
+                        const uint64_t val = (uint64_t)epoch0 + 1 + k;
+                        for (int t0 = k, c = 0; t0 < p; t0 += CH, ++c) {
+                            const int t1 = std::min(p, t0 + CH);
+                            CUDA_TRY(h, tqr::sig_wait_geq32(D.s_comm, O->flags + (int64_t)(t1 - 1) * (nb / ib) + nb / ib - 1,
+                                                            epoch0 + (unsigned)k + 1));
+                            CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_tiles[slot], t0 * vt), D.dev, h->at(src.V, t0 * vt),
+                                                            O->dev, es * (size_t)(t1 - t0) * vt, D.s_comm));
+                            CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_T[slot], t0 * tsz), D.dev, h->at(src.T, t0 * tsz),
+                                                            O->dev, es * (size_t)(t1 - t0) * tsz, D.s_comm));
+                            if (t0 == k)
+                                CUDA_TRY(h, cudaMemcpyPeerAsync(D.rb_V[slot], D.dev, src.Vexp, O->dev, es * (size_t)vt,
+                                                                D.s_comm));
+                            CUDA_TRY(h, tqr::sig_write(D.s_comm, reinterpret_cast<uint64_t*>(D.cflg) + slot * kMaxChunks + c, val));
+                        }
+                        CUDA_TRY(h, cudaEventRecord(D.ev_recv[k], D.s_comm));
+                        if (h->profile) {
+                            CUDA_TRY(h, cudaEventRecord(D.tb1[k], D.s_comm));
+                            D.tb_used[k] = 1;
+                            h->stats[3].flops += (double)es * ((p - k) * (vt + tsz) + vt);
+                        }
+                        continue;
+                    }
                     CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_tiles[slot], k * vt), D.dev, h->at(src.V, k * vt), O->dev,
                                                     es * (size_t)(p - k) * vt, D.s_comm));
                     CUDA_TRY(h, cudaMemcpyPeerAsync(h->at(D.rb_T[slot], k * tsz), D.dev, h->at(src.T, k * tsz), O->dev,
@@ -1659,16 +1750,28 @@ static tqr_status tqr_factor_tiles_impl(tqr_plan h) {
                 // dispatched first) and waits per reflector tile on the panel's flags; otherwise it
                 // follows the whole panel (or the broadcast) on the panel stream.
                 // (not with logical owners: several owners' lookaheads could then spin on one GPU)
-                const bool ovl = mine && h->la_overlap && h->la_fits && !h->logical && !h->f32() && h->ndom(k) == 1;
-                cudaStream_t sl = ovl ? D.s_look : D.s_panel;
-                if (!ovl) CUDA_TRY(h, cudaStreamWaitEvent(sl, ready, 0));
+                // logical owners share one GPU: the local overlap there too, behind the pre-panel event
+                // (at most one lookahead spins at a time, as for the remote trailing one)
+                const bool ovl = mine && h->la_overlap && h->la_fits && (!h->logical || h->la_remote) && !h->f32() &&
+                                 h->ndom(k) == 1;
+                // remote panel: trail its chunks (chunk flags of the receive slot) instead of the whole panel
+                const bool rtrail = !mine && h->la_remote && !h->f32() && h->ndom(k) == 1;
+                cudaStream_t sl = (ovl || rtrail) ? D.s_look : D.s_panel;
+                if (!ovl && !rtrail) CUDA_TRY(h, cudaStreamWaitEvent(sl, ready, 0));
+                if ((rtrail && O) || (ovl && h->logical))
+                    CUDA_TRY(h, cudaStreamWaitEvent(sl, O->ev_prepanel[k], 0));   // in-process root
                 if (k >= 1) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_u[stream_of(first, (int)D.cols.size())][k - 1], 0));
                 if (k == 0 && h->streamed) CUDA_TRY(h, cudaStreamWaitEvent(sl, D.ev_load[first], 0));
                 const int wl = w_look(h);
+                const unsigned long long* cf = nullptr;
+                if (rtrail)
+                    cf = h->ipc_mode ? reinterpret_cast<const unsigned long long*>(h->flags64 + F_CHUNK + slot * kMaxChunks)
+                                     : D.cflg + slot * kMaxChunks;
                 CUDA_TRY(h, update(h, r, D.tiles, colsz, tile, nb, first, 1, k, wl, nb / wl, true, sl,
-                                   &h->launches, ovl ? D.flags : nullptr, epoch0 + (unsigned)k + 1));
+                                   &h->launches, ovl ? D.flags : nullptr, epoch0 + (unsigned)k + 1,
+                                   cf, (unsigned long long)epoch0 + 1 + k, h->la_chunk));
                 emit(2, k, k, D.cols[first], ok);
-                if (ovl) {   // PANEL(k+1) (panel stream) after the lookahead
+                if (ovl || rtrail) {   // PANEL(k+1) (panel stream) after the lookahead
                     CUDA_TRY(h, cudaEventRecord(D.ev_look[k], sl));
                     CUDA_TRY(h, cudaStreamWaitEvent(D.s_panel, D.ev_look[k], 0));
                 }

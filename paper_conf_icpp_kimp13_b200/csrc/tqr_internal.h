@@ -65,6 +65,12 @@ struct UpdateArgsT {
     // i then is, by the panel's release/acquire chain); null = the stream dependency suffices
     const unsigned* wflags = nullptr;
     unsigned wepoch = 0;
+    // Lookahead trailing a REMOTE panel (another owner's): before reading reflector tile i, wait
+    // until the chunk flag cflags[(i - k) / cchunk] (64-bit, in this owner's memory, raised by the
+    // transfer of that chunk of tiles into the receive slot) is >= cval; null = not trailing
+    const unsigned long long* cflags = nullptr;
+    unsigned long long cval = 0;
+    int cchunk = 1;
     // FP64 wavefront apply of nsteps consecutive panels in one launch (tqr_apply_qt / solve_ls,
     // single owner, flat tree): grid = nsteps * nslc CTAs, step offset st = CTA / nslc processes
     // step k +- st (TRANS: +) with V, T, Vexp advanced by st * (vcol, tcol, ecol) elements; prog
@@ -122,6 +128,8 @@ int64_t f32_img_tile(int nb, int ib);
 cudaError_t sig_write(cudaStream_t s, uint64_t* addr, uint64_t v);
 // later work of s waits until (int64_t)(*addr - v) >= 0 (addr: this process's device memory)
 cudaError_t sig_wait_geq(cudaStream_t s, const uint64_t* addr, uint64_t v);
+// 32-bit variant (the panel kernel's publication flags): later work waits until (int32_t)(*addr - v) >= 0
+cudaError_t sig_wait_geq32(cudaStream_t s, const unsigned* addr, unsigned v);
 bool signal_uses_memops();
 size_t panel_smem_bytes(int nb, int ib);
 size_t update_smem_bytes(int nb, int ib, int w);

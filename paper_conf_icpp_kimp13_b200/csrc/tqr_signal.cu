@@ -26,11 +26,13 @@ namespace {
 
 using WaitFn = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 using WriteFn = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+using Wait32Fn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 
 struct MemOps {
     bool tried = false;
     WaitFn wait = nullptr;
     WriteFn write = nullptr;
+    Wait32Fn wait32 = nullptr;
 };
 
 MemOps& memops() {
@@ -47,6 +49,11 @@ MemOps& memops() {
             q1 == cudaDriverEntryPointSuccess && q2 == cudaDriverEntryPointSuccess && fw && fr) {
             m.wait = reinterpret_cast<WaitFn>(fw);
             m.write = reinterpret_cast<WriteFn>(fr);
+            void* f32 = nullptr;
+            cudaDriverEntryPointQueryResult q3 = cudaDriverEntryPointSymbolNotFound;
+            if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &f32, cudaEnableDefault, &q3) == cudaSuccess &&
+                q3 == cudaDriverEntryPointSuccess && f32)
+                m.wait32 = reinterpret_cast<Wait32Fn>(f32);
         }
         cudaGetLastError();
     }
@@ -70,9 +77,31 @@ __global__ void sig_wait_kernel(const uint64_t* addr, uint64_t v) {
     }
 }
 
+__global__ void sig_wait32_kernel(const unsigned* addr, unsigned v) {
+    if (threadIdx.x == 0) {
+        for (;;) {
+            unsigned x;
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(x) : "l"(addr) : "memory");
+            if ((int)(x - v) >= 0) break;
+            __nanosleep(256);
+        }
+        __threadfence_system();
+    }
+}
+
 }  // namespace
 
 bool signal_uses_memops() { return memops().wait != nullptr; }
+
+cudaError_t sig_wait_geq32(cudaStream_t s, const unsigned* addr, unsigned v) {
+    MemOps& m = memops();
+    if (m.wait32) {
+        return m.wait32((CUstream)s, (CUdeviceptr)addr, (cuuint32_t)v, CU_STREAM_WAIT_VALUE_GEQ) == CUDA_SUCCESS
+                   ? cudaSuccess : cudaErrorUnknown;
+    }
+    sig_wait32_kernel<<<1, 32, 0, s>>>(addr, v);
+    return cudaGetLastError();
+}
 
 cudaError_t sig_write(cudaStream_t s, uint64_t* addr, uint64_t v) {
     MemOps& m = memops();
