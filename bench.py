@@ -387,7 +387,9 @@ def main():
         cpu = {"value": round(v, 3), "unit": "GFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
                "sample": desc}
         # the oracle on one thread as well (a narrower sample: ~1-3 s of host work)
-        v1, dt1, desc1 = oracle_sample(args.config, nthreads=1, ncols=min(256, CONFIGS[args.config][1]))
+        mm, nn = CONFIGS[args.config][0], CONFIGS[args.config][1]
+        ns1 = int(min(256, nn, max(32, (2e10 / mm) ** 0.5)))      # <= ~2e10 flops of 1-thread work
+        v1, dt1, desc1 = oracle_sample(args.config, nthreads=1, ncols=ns1)
         cpu["single_thread"] = {"value": round(v1, 3), "unit": "GFLOP/s", "cores": 1, "sample": desc1}
 
     if rank == 0:

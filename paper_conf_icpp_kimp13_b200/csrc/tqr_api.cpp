@@ -759,8 +759,10 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
     // Panel sub-slicing: split the apply chain of each ib column block over 4 CTAs when the
     // panel is on the critical path (few trailing columns per panel step or several owners).
     // measured (r02): 4 sub-slices (W = 8) cut the C5 8-owner critical path 417 -> 345 ms and C3
-    // 236.9 -> 232.1 ms; the last column blocks' sequential applies bound the TS wavefront
-    h->panel_split = 4;
+    // 236.9 -> 232.1 ms (the last column blocks' sequential applies bound the TS wavefront); a single
+    // owner with many columns (C5 on one GPU: panels hidden behind the updates) keeps 2 (1640 vs 1646 ms:
+    // fewer SMs taken from the bulk update)
+    h->panel_split = (ndev == 1 && h->q > 32) ? 2 : 4;
     if (ib < 32 && h->panel_split > 2) h->panel_split = 2;
     if (const char* e = getenv("TQR_PANEL_SPLIT")) { int v = atoi(e); if (v == 1 || v == 2 || v == 4) h->panel_split = v; }
     if (ib / h->panel_split < 8) h->panel_split = 1;
@@ -1018,9 +1020,12 @@ static tqr_status tqr_ipc_connect_impl(tqr_plan h, const void* all, int64_t len)
     }
     // ranks sharing a GPU are time-sliced: a lookahead spinning on another rank's chunk flags would
     // hold its context's slice -- no remote trailing then (same decision on every rank: all devices known)
-    for (int a = 0; a < h->world; ++a)
-        for (int b = a + 1; b < h->world; ++b)
-            if (std::memcmp(h->peers[a].uuid, h->peers[b].uuid, sizeof(h->peers[a].uuid)) == 0) h->la_remote = false;
+    // (TQR_LA_REMOTE=2 forces it anyway: the multi-process tests exercise the chunked IPC path on one GPU)
+    const char* lr = getenv("TQR_LA_REMOTE");
+    if (!(lr && atoi(lr) == 2))
+        for (int a = 0; a < h->world; ++a)
+            for (int b = a + 1; b < h->world; ++b)
+                if (std::memcmp(h->peers[a].uuid, h->peers[b].uuid, sizeof(h->peers[a].uuid)) == 0) h->la_remote = false;
     // arm: my receive slots 0 / 1 are free for steps 0 / 1 of the first factorization, at every
     // possible root (the flag lives in the root's block; roots only ever wait on their own block)
     cudaStream_t s = plan_comm_stream(h);

@@ -35,12 +35,12 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _run(tmp_path, world, m, n, nb, ib, dts="f64", guide=None, tree=-1, rs=0):
+def _run(tmp_path, world, m, n, nb, ib, dts="f64", guide=None, tree=-1, rs=0, env=None):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes", "1", "--nproc-per-node", str(world),
            "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
            os.path.join(ROOT, "tests", "mp_ipc_worker.py"), str(tmp_path), str(m), str(n), str(nb), str(ib), dts,
            "-" if guide is None else ",".join(map(str, guide)), str(tree), str(rs)]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT, env=dict(os.environ, **(env or {})))
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     return [dict(np.load(os.path.join(tmp_path, "rank%d.npz" % k))) for k in range(world)]
 
@@ -141,3 +141,17 @@ def test_multiprocess_ipc_row_split(tmp_path, world, m, n, nb, ib):
     Rl = Ad.cpu().numpy()
     plan.close()
     assert np.array_equal(np.triu(outs[0]["R0"][:n]), np.triu(Rl[:n]))
+
+
+def test_multiprocess_ipc_remote_trailing_chunks(tmp_path):
+    """The chunked IPC transfer + trailing lookahead (default on distinct GPUs) forced on the shared
+    test GPU (TQR_LA_REMOTE=2): chunk c of panel k is copied once the panel published its last tile
+    and raises a chunk flag the next owner's lookahead kernel waits on.  Bitwise the single-owner R."""
+    world, m, n, nb, ib = 2, 2048, 2048, 256, 32
+    outs = _run(tmp_path, world, m, n, nb, ib, "f64", None, -1, 0, env={"TQR_LA_REMOTE": "2"})
+    A = synthetic.gaussian(m, n, 9000 + m + n)
+    R1 = _single_owner(A, nb, ib, tqr.TQR_F64)
+    for key in ("R0", "R1", "Rhost"):
+        R = _assemble_cols(outs, key, lambda j: j % world, nb, n)
+        assert np.array_equal(R, R1), key
+    assert colnorm_rel_err(np.triu(R1[:n]), oracle.qr(A).R) <= 1e-10
