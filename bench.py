@@ -202,10 +202,11 @@ def main():
     ap.add_argument("--no-lookahead", action="store_true")
     ap.add_argument("--tree", type=int, default=0,
                     help="elimination tree: 0 auto (tree for q == 1), -1 flat TS, L > 0 TS domains of L tiles")
-    ap.add_argument("--guide", default="auto", choices=["auto", "cyclic", "pairs"],
+    ap.add_argument("--guide", default="auto", choices=["auto", "cyclic", "pairs", "snake"],
                     help="N > 1 column distribution (Eq. 12 guide array): cyclic {0..N-1}; pairs "
-                         "{0,0,1,1,..}: the lookahead column is local every other step; auto = pairs "
-                         "for N >= 8 (critical-path bound), cyclic otherwise")
+                         "{0,0,1,1,..}; snake {0..N-1, N-1..0} (balances the trailing work, which grows "
+                         "with the column index: max/mean per-GPU work 1.008 at C5 on 8 GPUs vs 1.082 "
+                         "cyclic and 1.158 pairs); auto = snake")
     ap.add_argument("--solve", type=int, default=0,
                     help="also time tqr_solve_ls with this many right-hand sides (NEXT-3; 'solve' key)")
     ap.add_argument("--tree-group", type=int, default=0,
@@ -264,8 +265,13 @@ def main():
         obj = [tqr.tqr_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         nccl_id = obj[0]
-    gmode = args.guide if args.guide != "auto" else ("pairs" if world >= 8 else "cyclic")
-    guide = [d for d in range(world) for _ in range(2 if gmode == "pairs" else 1)]
+    gmode = args.guide if args.guide != "auto" else "snake"
+    if world == 1:
+        guide = [0]
+    elif gmode == "snake":
+        guide = list(range(world)) + list(range(world - 1, -1, -1))
+    else:
+        guide = [d for d in range(world) for _ in range(2 if gmode == "pairs" else 1)]
     plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32 if f32 else tqr.TQR_F64, ndev=world, guide=guide,
                     rank=rank, world=world, nccl_id=nccl_id,
                     transport=("nccl" if args.transport == "nccl" else "ipc") if world > 1 else "auto",

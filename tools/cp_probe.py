@@ -18,7 +18,8 @@ m, n, nb, ib, seed = CONFIGS[cfg]
 g = torch.Generator(device="cuda").manual_seed(seed)
 A0 = torch.randn((n, m), dtype=torch.float64, device="cuda", generator=g).t()
 guides = {"cyclic": list(range(G)), "pairs": [d for d in range(G) for _ in range(2)],
-          "quads": [d for d in range(G) for _ in range(4)]}
+          "quads": [d for d in range(G) for _ in range(4)],
+          "snake": list(range(G)) + list(range(G - 1, -1, -1))}
 for name, guide in guides.items():
     plan = tqr.Plan(m, n, nb, ib, ndev=G, guide=guide, logical_devices=True)
     plan.load(A0)
