@@ -1,6 +1,7 @@
 """CPU-only checks of the C-ABI library: it loads, exports every symbol include/tqr.h
 declares, and its pure host logic (guide array, schedule, argument validation) is right.
 No compute calls are made here (no GPU in this container)."""
+import ctypes
 import os
 import re
 
@@ -158,3 +159,24 @@ def test_select_matches_oracle(L, seed):
     lo, Tpo, pbo = ds.num_dev_selection(M, N, T, 8, times, speed, main)
     assert order == lo and pb == pbo
     np.testing.assert_allclose(Tp, Tpo, rtol=1e-12)
+
+
+def test_guide_and_selection_bounded_on_extreme_rates(L):
+    """a guide longer than the cap (2^20 entries) is TQR_ERR_ARG, not an overflowed
+    length or a huge allocation; the device-count model clamps wildly mismatched rates."""
+    with pytest.raises(tqr.TqrError) as e:
+        tqr.tqr_generate_guide([2 ** 30, 1])
+    assert e.value.status == 1
+    assert len(tqr.tqr_generate_guide([2 ** 19, 2 ** 19 + 2])) == 2 ** 18 + 2 ** 18 + 1
+    times = [(1e-3, 1e-3, 1e-12, 1e-12), (1e-3, 1e-3, 1e3, 1e3)]     # update speeds 1e15 apart
+    order, tp, pb = tqr.tqr_select_ndev(4, 4, 64, 8, times, [[0, 1e9], [1e9, 0]], 0)
+    assert pb in (1, 2) and len(tp) == 2 and all(x > 0 for x in tp)
+
+
+def test_plan_queries_without_gpu(L):
+    """The plan-query entry points are NULL-safe (no GPU needed)."""
+    assert L.tqr_plan_flags(None) == 0
+    assert L.tqr_owner(None, 0) == -1
+    cnt = ctypes.c_int64()
+    assert L.tqr_issued_ops(None, None, 0, ctypes.byref(cnt)) == 1
+    assert L.tqr_ipc_handle(None, None, 0, ctypes.byref(cnt)) == 1
