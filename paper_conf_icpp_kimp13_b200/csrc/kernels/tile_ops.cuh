@@ -249,6 +249,7 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
     for (int h = 0; h < 2; ++h) {
         mbar_wait(&sm.mbar[wq][h], (vph >> h) & 1u);
         vph ^= 1u << h;
+        TQR_PH(h == 0 ? 5 : 11);                  // (probe) staging wait of V half h
         const double* vh = &sm.Vst[wq][h][0][0];
         double cp[NP][G::MF][G::JC][2];
 #pragma unroll
@@ -333,7 +334,61 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
     //      The A operand (W^T fragment) is summed from the partial slots as it is loaded; each
     //      warp owns fragments with one column block mf so it sums that A operand once.
     //      Wsm = -W' (GEMM2 operand); top -= W' written straight from the fragments.
-    {
+    if constexpr (SM::NSLOT == 8) {
+        // 8 slots (update kernel): reduce-scatter of the slots (+ top) into Wsm = W -- every
+        // element read once, 16-byte pairs, eight consecutive threads on 128 contiguous bytes --
+        // then the T multiply with A from Wsm (one load per k-step instead of nine) and the k-steps
+        // past a fragment's triangle skipped (exact zeros); -W' overwrites Wsm after a barrier.
+        // (Same sum order and products as the fused form below, which the 4-slot panel keeps.)
+        constexpr int NPAIR = W * IB / 2;
+        for (int idx = tid; idx < NPAIR; idx += kThreads) {
+            const int col = idx / (IB / 2), ib = 2 * (idx % (IB / 2));
+            double2 sv = top ? ld2(&sm.topsm[col * G::LDW + ib]) : make_double2(0.0, 0.0);
+#pragma unroll
+            for (int sl = 0; sl < SM::NSLOT; ++sl) {
+                const double2 pv = ld2(&sm.red[sl * (W * G::LDR) + col * G::LDR + ib]);
+                sv.x += pv.x;
+                sv.y += pv.y;
+            }
+            st2(&sm.Wsm[col * G::LDW + ib], sv.x, sv.y);
+        }
+        __syncthreads();
+        constexpr int NFRAG = G::MF * G::JF;
+        constexpr int FPW = (NFRAG + kWarps - 1) / kWarps;
+        const int f0 = wq * FPW, mf = f0 / G::JF;
+        double acc0[FPW][2], acc1[FPW][2];
+#pragma unroll
+        for (int u = 0; u < FPW; ++u) acc0[u][0] = acc0[u][1] = acc1[u][0] = acc1[u][1] = 0.0;
+        if (wq * FPW < NFRAG) {
+#pragma unroll
+            for (int kk = 0; kk < IB; kk += 4) {
+                const double av = sm.Wsm[(mf * 8 + g) * G::LDW + kk + t];
+#pragma unroll
+                for (int u = 0; u < FPW; ++u) {
+                    const int jf = (f0 + u) % G::JF;
+                    if (TRANS && kk >= jf * 8 + 8) continue;
+                    if (!TRANS && kk + 4 <= jf * 8) continue;
+                    double bv;
+                    if constexpr (TRANS) bv = sm.Traw[(jf * 8 + g) * G::LDT2 + kk + t];
+                    else                 bv = sm.Traw[(kk + t) * G::LDT2 + jf * 8 + g];
+                    if ((kk >> 2) & 1) dmma(acc1[u][0], acc1[u][1], av, bv);
+                    else               dmma(acc0[u][0], acc0[u][1], av, bv);
+                }
+            }
+        }
+        __syncthreads();
+        if (wq * FPW < NFRAG) {
+#pragma unroll
+            for (int u = 0; u < FPW; ++u) {
+                const int jf = (f0 + u) % G::JF;
+                const double w0 = acc0[u][0] + acc1[u][0], w1 = acc0[u][1] + acc1[u][1];
+                const int col = mf * 8 + g, r = jf * 8 + 2 * t;
+                st2(&sm.Wsm[col * G::LDW + r], -w0, -w1);
+                if (top) st2(top + (int64_t)col * ldtop + r, sm.topsm[col * G::LDW + r] - w0,
+                             sm.topsm[col * G::LDW + r + 1] - w1);
+            }
+        }
+    } else {
         constexpr int NFRAG = G::MF * G::JF;
         constexpr int FPW = (NFRAG + kWarps - 1) / kWarps;   // fragments per warp (JF % FPW == 0)
         static_assert(NFRAG <= kWarps || G::JF % FPW == 0, "fragment assignment");

@@ -164,9 +164,10 @@ struct tqr_plan_s {
     int nstreams_io = 8;            // streamed factor: contiguous column chunks, one stream each
     int nstreams_alloc() const { return std::max(nstreams, nstreams_io); }
     int panel_split = 1;            // sub-slice CTAs per ib column block in the panel kernel
+    int w_look = 0;                 // lookahead slice width (0 = default: 8 at nb >= 256, else 16)
     int tree_L = 0;                 // TS-domain length (tiles); 0 = flat TS chain
     int dmax = 1;                   // max domains of any step = ceil(p / tree_L)
-    int tree_G = 0;                 // two-level merge: groups of G domains (0 = one flat merge chain)
+    int tree_G = 0;                 // merge tree: groups of G heads per level (0 = one flat merge chain)
     int merge_split = 1;            // panel sub-slice split of the level-1 merge jobs
     // streamed tqr_factor (caller A not on the owner's device): column loads overlap the
     // factorization (panel k / the step-0 update of column j wait for ev_load), R of column k is
@@ -183,7 +184,9 @@ struct tqr_plan_s {
                                     // bulk updates -> panels + lookahead only = the critical path
     void* sA = nullptr;
     int64_t slda = 0;
-    int ngroups(int D) const { return (tree_G > 1 && D > tree_G) ? (D + tree_G - 1) / tree_G : 1; }
+    // merge tree of D domain heads: level l merges, in groups of G consecutive heads of stride G^l,
+    // heads gG+1..gG+G-1 into head gG (one multi-job launch per level); G >= D: one flat chain
+    int merge_group(int D) const { return tree_G > 1 ? tree_G : std::max(2, D); }
     int ndom(int k) const { return tree_L > 0 ? (p - k + tree_L - 1) / tree_L : 1; }
     bool tree_one_cta = true;       // domain phase: one CTA per domain (long domains) or wavefront jobs
     int tree_split = 1;             // panel split of the wavefront domain jobs
@@ -278,7 +281,10 @@ bool supported_nb_ib(int nb, int ib) {
 
 // Slice width of the bulk update kernel and of the (latency-critical) lookahead column.
 int w_bulk(const tqr_plan_s*) { return 32; }
-int w_look(const tqr_plan_s* h) { return h->nb >= 256 ? 8 : 16; }
+int w_look(const tqr_plan_s* h) {
+    if (h->w_look > 0) return h->w_look;
+    return h->nb >= 256 ? 8 : 16;
+}
 
 double flops_update(const tqr_plan_s* h, int k, int ncols) {
     const double nb3 = (double)h->nb * h->nb * h->nb;
@@ -718,6 +724,7 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_LA_OVERLAP")) h->la_overlap = atoi(e) != 0;
     if (const char* e = getenv("TQR_CRITICAL_PATH_PROBE")) h->cp_probe = atoi(e) != 0;
+    if (const char* e = getenv("TQR_W_LOOK")) { int v = atoi(e); if (v == 8 || v == 16 || v == 32) h->w_look = v; }
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
     // Tree mode (NEXT-1): TS domains of L tiles factored one per CTA, merged by a flat TT chain.
     // Auto: a single panel column (q == 1, e.g. C4) whose flat chain has parallelism 1.
@@ -744,8 +751,8 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
     }
     if (h->tree_L > 0 && dtype != TQR_F64) { h->tree_L = 0; if (o.tree_domain > 0) { delete h; return fail(nullptr, TQR_ERR_UNSUPPORTED, "tree mode: FP64 only in this build"); } }
     h->dmax = h->ndom(0);
-    // Two-level merge of the D domain heads: groups of G ~ sqrt(D) merged concurrently, then the
-    // group heads (D - 1 sequential merges -> G - 1 + ceil(D/G) - 1).
+    // Merge tree of the D domain heads: per level, groups of G heads merged concurrently (D - 1
+    // sequential merges -> (G - 1) * ceil(log_G D)); default G ~ sqrt(D) (two levels).
     if (h->tree_L > 0) {
         const int D0 = h->dmax;
         if (o.tree_group > 1) h->tree_G = o.tree_group;
@@ -773,7 +780,7 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
         int sms = 148;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
         const int panel_ctas = (nb / ib) * (h->panel_split + 1);
-        const int look_ctas = nb / (nb >= 256 ? 8 : 16);
+        const int look_ctas = nb / w_look(h);
         h->la_fits = panel_ctas + look_ctas <= sms;
     }
     {
@@ -1176,39 +1183,23 @@ cudaError_t update(const tqr_plan_s* h, const PanelRefs& r, void* X, int64_t col
         return update1(h, r.V, r.T, r.Vexp, X, col_stride, tile_stride, ld, group0, gstride, k, h->p, 1, w, nslices,
                        trans, s, 1, nullptr, 0, L, D);
     };
-    const int NG = h->ngroups(D), G = h->tree_G;
-    const int64_t tsz = (int64_t)h->ib * h->nb;
-    auto mrg = [&]() {   // flat merge chain
-        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L, ld, group0,
-                       gstride, 0, D, 0, w, nslices, trans, s);
+    // merge level of stride S (heads 0, S, 2S, .. of the domain heads, row tiles k + i*S*L, merge
+    // slots i*S): jobs of G consecutive heads, each the chain of heads gG+1.. against head gG
+    const int G = h->merge_group(D);
+    std::vector<int64_t> lv;
+    for (int64_t S = 1; S < D; S *= G) lv.push_back(S);
+    auto level = [&](int64_t S) {
+        const int H = (int)((D + S - 1) / S), nj = (H + G - 1) / G;
+        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L * S, ld,
+                       group0, gstride, 0, H, 0, w, nslices, trans, s, (int)S, nullptr, 0, nj > 1 ? G : 0, nj);
     };
-    // level 1: every group's chain against its head gG in one launch (jobs of G merge slots)
-    auto grps = [&]() {
-        (void)tsz;
-        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L, ld, group0,
-                       gstride, 0, D, 0, w, nslices, trans, s, 1, nullptr, 0, G, NG);
-    };
-    auto top = [&]() {   // level 2: group heads G, 2G, .. against head 0 (merge slots stride G)
-        return update1(h, r.M, r.MT, r.M, h->at(X, (int64_t)k * tile_stride), col_stride, tile_stride * L * G, ld,
-                       group0, gstride, 0, NG, 0, w, nslices, trans, s, G);
-    };
-    if (nl) *nl += (NG > 1 ? 3 : 2);
+    if (nl) *nl += 1 + (int64_t)lv.size();
     cudaError_t e = cudaSuccess;
-    if (trans) {
+    if (trans) {   // Q^T: domains, then the merge levels bottom-up
         e = doms();
-        if (NG == 1) {
-            if (e == cudaSuccess) e = mrg();
-        } else {
-            if (e == cudaSuccess) e = grps();
-            if (e == cudaSuccess) e = top();
-        }
-    } else {
-        if (NG == 1) {
-            e = mrg();
-        } else {
-            e = top();
-            if (e == cudaSuccess) e = grps();
-        }
+        for (size_t l = 0; l < lv.size() && e == cudaSuccess; ++l) e = level(lv[l]);
+    } else {       // Q: the merge levels top-down, then the domains
+        for (size_t l = lv.size(); l-- > 0 && e == cudaSuccess;) e = level(lv[l]);
         if (e == cudaSuccess) e = doms();
     }
     return e;
@@ -1457,22 +1448,20 @@ tqr_status launch_panel_step(tqr_plan h, Owner& O, int k, unsigned epoch) {
         m.skip_ge = 1;
         m.flags = O.mflags;
         m.fslots = p;
-        const int NG = h->ngroups(D);
-        if (NG == 1) {
-            CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m, O.s_panel));
-            h->launches += 3;
-            return TQR_OK;
+        // merge tree, one launch per level of stride S: H = ceil(D/S) heads (slots 0, S, 2S, ..), jobs
+        // of G consecutive heads -- job g merges heads gG+1..gG+G-1 into head gG (job 0's top is the
+        // real head tile, job g > 0's is merge slot gGS); a single job is one chain (split as a panel)
+        const int G = h->merge_group(D);
+        int nlv = 0;
+        for (int64_t S = 1; S < D; S *= G, ++nlv) {
+            const int H = (int)((D + S - 1) / S), nj = (H + G - 1) / G;
+            tqr::PanelArgs ml = m;
+            ml.stride = (int)S;
+            ml.p = H;
+            ml.L = nj > 1 ? G : 0;
+            CUDA_TRY(h, tqr::launch_panel(nb, ib, nj > 1 ? h->merge_split : h->panel_split, ml, O.s_panel, nj));
         }
-        // two-level merge: NG concurrent chains (job g merges heads gG+1.. into head gG; job 0's
-        // top is the real head tile, job g > 0's is merge slot gG), then the chain of group heads
-        tqr::PanelArgs m1 = m;
-        m1.L = h->tree_G;
-        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->merge_split, m1, O.s_panel, NG));
-        tqr::PanelArgs m2 = m;
-        m2.stride = h->tree_G;
-        m2.p = NG;
-        CUDA_TRY(h, tqr::launch_panel(nb, ib, h->panel_split, m2, O.s_panel));
-        h->launches += 4;
+        h->launches += 2 + nlv;
         return TQR_OK;
     }
     CUDA_TRY(h, tqr::launch_widen(h->at<float>(O.tiles, lc * colsz + k * tile), O.sc_col + k * tile,

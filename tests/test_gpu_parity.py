@@ -616,8 +616,12 @@ def test_tree_matches_oracle(m, n, nb, ib, L, one_cta, monkeypatch):
 
 
 MERGES = [
-    # (m, n, nb, ib, L, G): two-level merge -- groups of G domain heads, then the group heads
+    # (m, n, nb, ib, L, G): merge tree -- per level, groups of G heads (G >= sqrt(D): two levels)
     (1024, 128, 64, 16, 1, 4),      # p=16: 16 domains -> 4 groups of 4 (step 1: 15 -> 4, last of 3)
+    (1024, 128, 64, 16, 1, 2),      # binary tree: 16 -> 8 -> 4 -> 2 -> 1 (step 1: 15 heads, odd levels)
+    (3000, 64, 64, 16, 1, 3),       # 47 heads, G=3: 47 -> 16 -> 6 -> 2 -> 1, ragged rows
+    (2048, 256, 64, 16, 2, 2),      # binary, ragged per step
+    (8192, 512, 512, 32, 1, 2),     # binary at nb=512, q=1
     (2048, 256, 64, 16, 2, 3),      # p=32, q=4: 16 -> 6 groups (last of 1 domain), ragged per step
     (1000, 300, 64, 16, 1, 5),      # ragged both ways
     (8192, 512, 512, 32, 2, 3),     # q=1 at nb=512: 8 domains -> groups 3,3,2
@@ -626,7 +630,7 @@ MERGES = [
 
 
 @pytest.mark.parametrize("m,n,nb,ib,L,G", MERGES)
-def test_two_level_merge_matches_oracle(m, n, nb, ib, L, G):
+def test_merge_tree_matches_oracle(m, n, nb, ib, L, G):
     A = synthetic.gaussian(m, n, 5300 + m + n + nb + L + G)
     plan, Rg = gpu_qr(A, nb, ib, tree_domain=L, tree_group=G)
     ref = oracle.qr(A)
@@ -642,7 +646,7 @@ def test_two_level_merge_matches_oracle(m, n, nb, ib, L, G):
     np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
     plan.close()
     # the flat merge chain reaches the same R (unique) and the logical-device partition replays
-    # the two-level tree through the broadcast path bitwise
+    # the merge tree through the broadcast path bitwise
     _, Rf = gpu_qr(A, nb, ib, tree_domain=L, tree_group=-1)
     assert colnorm_rel_err(np.triu(Rg[:n]), np.triu(Rf[:n])) <= R_TOL
     if n > nb:

@@ -21,8 +21,8 @@ with tqr.Plan(m, n, nb, ib) as p:
     p.load(A); p.factor_tiles(); p.store_r(R)
     torch.cuda.synchronize()
     L.tqr_probe_phases(buf, 0)
-names = ["T cp.async+top ld", "GEMM1 half A", "GEMM1 half B", "stage1 st+sync", "RMW+sync", "reduce+sync",
-         "T-DMMA+sync", "top store", "GEMM2 half A", "stage A", "GEMM2 half B", "stage B"]
+names = ["T cp.async+top ld", "GEMM1 half A", "GEMM1 half B", "stage1 st+sync", "RMW+sync", "wait V half A",
+         "T-DMMA+sync", "top store", "GEMM2 half A", "GEMM2 half B", "-", "wait V half B"]
 tot = sum(buf[i] for i in range(12))
 for i, nm in enumerate(names):
     print("%-20s %6.2f%%" % (nm, 100.0 * buf[i] / tot))
