@@ -23,9 +23,11 @@ SAN = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitize
 @pytest.mark.parametrize("tool", ["racecheck", "synccheck", "memcheck"])
 def test_sanitizer_clean(tool):
     out = subprocess.run([SAN, "--tool", tool, "--print-limit", "10", sys.executable,
-                          os.path.join(ROOT, "tools", "debug", "sanitize_run.py")],
+                          os.path.join(ROOT, "tools", "sanitize_run.py")],
                          cwd=ROOT, capture_output=True, text=True, timeout=900)
     text = out.stdout + out.stderr
+    if out.returncode == 86 and "closed" in text:   # the pool's wrapper refuses the tool (B200_PROFILING.md)
+        pytest.skip("compute-sanitizer is closed on this GPU pool: " + text.strip()[:200])
     assert out.returncode == 0, text[-3000:]
     assert "ok 1024 1024 512 32" in text and "ok extra" in text, text[-3000:]
     assert ("0 errors" in text) or ("0 hazards displayed (0 errors" in text), text[-3000:]
