@@ -416,10 +416,12 @@ def main():
                         "busy_ms_per_step": round(ums / K, 3), "share_of_step": round(ums / K / ms, 3)}
         else:
             # dominant kernel: the panel step (C4: one column -> the whole factorisation is panel
-            # work: TS-domain kernel + TT merge chain in tree mode, DMMA.8x8x4)
+            # work: TS-domain kernel + TT merge chain in tree mode; C1/C2: the flat panel wavefront)
             pach = pflops / max(pms, 1e-9) / 1e9
             roofline = {"bound": "alu" if f32 else "tensor",
-                        "kernel": "panel step (domain_kernel<%d,%d> + merge panel_kernel, DMMA.8x8x4)" % (nb, ib),
+                        "kernel": ("panel step (domain_kernel<%d,%d> + merge panel_kernel, DMMA.8x8x4)" % (nb, ib))
+                        if pflags & tqr.PLAN_TREE else
+                        ("panel_kernel<%d,%d> (GEQRT + flat TSQRT wavefront, factor_block + DMMA applies)" % (nb, ib)),
                         "achieved": round(pach, 3), "peak": peak, "unit": "TFLOP/s", "frac": round(pach / peak, 4),
                         "traffic": prof.get("dram_bytes_per_launch"), "traffic_note": prof.get("note"),
                         "peak_source": peak_src, "launches_per_step": pcount // K,
