@@ -197,6 +197,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"],
                     help="f32: the C5 FP32 configuration (FFMA updates)")
+    ap.add_argument("--ib", type=int, default=0,
+                    help="inner block ib (default: the config's; C3-C5 leave ib open, SURVEY 8)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-lookahead", action="store_true")
@@ -249,6 +251,8 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device("cuda", device))
 
     m, n, nb, ib, seed = CONFIGS[args.config]
+    if args.ib:
+        ib = args.ib
     f32 = args.dtype == "f32"
     tdt = torch.float32 if f32 else torch.float64
     es = 4 if f32 else 8
