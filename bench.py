@@ -412,7 +412,9 @@ def main():
             # dominant kernel: the bulk trailing update
             roofline = {"bound": "alu" if f32 else "tensor",
                         "kernel": "update_kernel32<%d,32,%d> (UNMQR+TSMQR chain, FFMA)" % (nb, ib) if f32 else
-                        "update_kernel<%d,32,%d> (UNMQR+TSMQR chain, DMMA.8x8x4)" % (nb, ib),
+                        ("update_kernel16<%d,%d> (UNMQR+TSMQR chain, 16 warps, DMMA.8x8x4)" % (nb, ib)
+                         if nb >= 256 and os.environ.get("TQR_W16", "1") != "0" else
+                         "update_kernel<%d,32,%d> (UNMQR+TSMQR chain, DMMA.8x8x4)" % (nb, ib)),
                         "achieved": round(achieved, 3), "peak": peak, "unit": "TFLOP/s",
                         "frac": round(achieved / peak, 4),
                         "traffic": prof.get("dram_bytes_per_launch"), "traffic_note": prof.get("note"),

@@ -175,6 +175,7 @@ struct tqr_plan_s {
     void* prog = nullptr;           // wavefront apply progress flags (q * nslices)
     size_t prog_n = 0;
     bool la_overlap = true;         // FP64 flat lookahead runs beside PANEL(k) on per-tile flags
+    bool w16 = true;                // FP64 bulk Q^T chains on 16 warps per CTA (TQR_W16=0: 8 warps)
     bool la_fits = true;            // ... only when its spinning CTAs leave SMs for the whole panel grid
     bool la_remote = false;         // the lookahead of column k+1 on ANOTHER owner trails PANEL(k) chunk by chunk
     int la_chunk = 8;               // tiles per trailing transfer chunk
@@ -723,6 +724,7 @@ static tqr_status tqr_create_ex_impl(int64_t m, int64_t n, int32_t nb, int32_t i
     h->lookahead = o.no_lookahead == 0;
     h->profile = o.profile != 0;
     if (const char* e = getenv("TQR_LA_OVERLAP")) h->la_overlap = atoi(e) != 0;
+    if (const char* e = getenv("TQR_W16")) h->w16 = atoi(e) != 0;
     if (const char* e = getenv("TQR_CRITICAL_PATH_PROBE")) h->cp_probe = atoi(e) != 0;
     if (const char* e = getenv("TQR_W_LOOK")) { int v = atoi(e); if (v == 8 || v == 16 || v == 32) h->w_look = v; }
     if (const char* e = getenv("TQR_UPDATE_STREAMS")) { int v = atoi(e); if (v >= 1 && v <= 16) h->nstreams = v; }
@@ -1158,6 +1160,7 @@ cudaError_t update1(const tqr_plan_s* h, const void* V, const void* T, const voi
     u.group0 = group0; u.gstride = gstride; u.k = k_head; u.p = p_end; u.do_unmqr = do_unmqr; u.vstride = vstride;
     u.wflags = wflags; u.wepoch = wepoch;
     u.cflags = cflags; u.cval = cval; u.cchunk = cchunk;
+    u.w16 = h->w16 ? 1 : 0;
     if (domL > 0) { u.domL = domL; u.nslc = nslices; }
     return tqr::launch_update(h->nb, h->ib, w, u, nslices * njobs, trans, s);
 }

@@ -80,6 +80,9 @@ struct UpdateArgsT {
     int domL = 0;                        // > 0: tree jobs of domL row tiles (see update_kernel)
     int64_t vcol = 0, tcol = 0, ecol = 0;
     unsigned* prog = nullptr;
+    // FP64, W = 32, nb >= 256, plain Q^T chain: run update_kernel16 (the slice over 16 warps,
+    // tile_w16.cuh) instead of the 8-warp update_kernel
+    int w16 = 0;
 };
 using UpdateArgs = UpdateArgsT<double>;
 
