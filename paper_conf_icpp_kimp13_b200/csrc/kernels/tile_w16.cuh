@@ -25,8 +25,9 @@ struct Smem16 {
     using G = Geom<NB, 32, IB>;              // RW = NB/8 rows per row group, HC, LDR, LDW, LDT2
     uint64_t mbar[8][2];                     // [row group][half]
     double Vst[8][2][G::HC][G::RW];          // [row group][half], layout of vst_off
-    double red[2 * 8 * 16 * G::LDR];         // [cg][rg][col 0..15][ib] partial slots
-    double Wsm[32 * G::LDW];                 // W (reduce-scatter), then -W' (GEMM2 operand)
+    double red[2 * 8 * 16 * G::LDR];         // [cg][rg][col 0..15][ib] partial slots; the 4 pad doubles
+                                             // of each slot column hold -W' (GEMM2 operand), wsm_off
+    double Wsm[32 * G::LDW];                 // W (reduce-scatter)
     double Traw[IB * G::LDT2];               // T(r', r) at r*LDT2 + r'
     double topsm[32 * G::LDW];               // X1 rows (r, c) at c*LDW + r
 };
@@ -56,6 +57,15 @@ struct Slice16 {
                 st2(P + (int64_t)(c0() + mf * 8) * ld + r0() + nf * 8, acc[mf][nf][0], acc[mf][nf][1]);
     }
 };
+
+// -W'(col, r) in the padding of the partial slots (ib 32..35 of slot (col / 16, r / 4), column
+// col % 16): no partial store ever writes there, so the next block's GEMM1 stores cannot race with
+// a slower warp's GEMM2 reads, and the T multiply can write it without a barrier after its reads
+// of Wsm.  Lanes (g, t) of an A-fragment load hit banks (4g + t) mod 16: two wavefronts.
+template <int LDR>
+__device__ __forceinline__ int wsm_off(int col, int r) {
+    return ((col >> 4) * 8 + (r >> 2)) * (16 * LDR) + (col & 15) * LDR + (LDR - 4) + (r & 3);
+}
 
 __device__ __forceinline__ void pair_sync(int rg) {   // the two warps of row group rg
     asm volatile("bar.sync %0, 64;" ::"r"(1 + rg) : "memory");
@@ -165,11 +175,10 @@ __device__ __forceinline__ void apply_block16(Slice16<NB, IB>& X, Smem16<NB, IB>
             else               dmma(w0, w1, av, bv);
         }
     }
-    __syncthreads();
     if (wl < NFRAG) {
         const int col = fmf * 8 + g, r = fjf * 8 + 2 * t;
         const double a0 = w0 + v0, a1 = w1 + v1;
-        st2(&sm.Wsm[col * G::LDW + r], -a0, -a1);
+        st2(&sm.red[wsm_off<G::LDR>(col, r)], -a0, -a1);   // r even: r, r+1 in one 16-byte pair
         if (top) st2(top + (int64_t)col * ldtop + r, sm.topsm[col * G::LDW + r] - a0, sm.topsm[col * G::LDW + r + 1] - a1);
     }
     __syncthreads();
@@ -185,7 +194,7 @@ __device__ __forceinline__ void apply_block16(Slice16<NB, IB>& X, Smem16<NB, IB>
         for (int kk = 0; kk < HC; kk += 4) {
             double a[2];
 #pragma unroll
-            for (int mf = 0; mf < 2; ++mf) a[mf] = sm.Wsm[(cg * 16 + mf * 8 + g) * G::LDW + h * HC + kk + t];
+            for (int mf = 0; mf < 2; ++mf) a[mf] = sm.red[wsm_off<G::LDR>(cg * 16 + mf * 8 + g, h * HC + kk + t)];
 #pragma unroll
             for (int nf = 0; nf < NF; ++nf) {
                 if (KM && rbase + nf * 8 + 8 <= kmin) continue;
