@@ -214,6 +214,10 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
     const int lane = lane_id(), g = lane >> 2, t = lane & 3, wq = warp_id();
     const int rbase = wq * G::RW;
     const int tid = threadIdx.x;
+    // 8 slots: -W'(col, r) lives in the 4 padding doubles (ib IB..IB+3) of slot r/4, column col;
+    // A-fragment loads hit banks (4g + t) mod 16 (two wavefronts)
+    static_assert(SM::NSLOT != 8 || G::LDR - IB == 4 && IB <= 4 * SM::NSLOT, "padding holds -W'");
+    auto pad_off = [](int col, int r) { return (r >> 2) * (W * G::LDR) + col * G::LDR + IB + (r & 3); };
     TQR_PH0();
 
     // ---- (0) half B of V (bulk), T block and top rows (LDGSTS group, waited before barrier 1)
@@ -376,14 +380,15 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
                 }
             }
         }
-        __syncthreads();
+        // -W' goes to the padding of the partial slots (pad_off), which no GEMM1 store writes, so no
+        // barrier is needed between the reads of Wsm above and these writes
         if (wq * FPW < NFRAG) {
 #pragma unroll
             for (int u = 0; u < FPW; ++u) {
                 const int jf = (f0 + u) % G::JF;
                 const double w0 = acc0[u][0] + acc1[u][0], w1 = acc0[u][1] + acc1[u][1];
                 const int col = mf * 8 + g, r = jf * 8 + 2 * t;
-                st2(&sm.Wsm[col * G::LDW + r], -w0, -w1);
+                st2(&sm.red[pad_off(col, r)], -w0, -w1);
                 if (top) st2(top + (int64_t)col * ldtop + r, sm.topsm[col * G::LDW + r] - w0,
                              sm.topsm[col * G::LDW + r + 1] - w1);
             }
@@ -439,7 +444,9 @@ __device__ __forceinline__ void apply_block(Slice<NB, W, IB>& X, Smem<NB, W, IB,
         for (int kk = 0; kk < G::HC; kk += 4) {
             double a[G::MF];
 #pragma unroll
-            for (int mf = 0; mf < G::MF; ++mf) a[mf] = sm.Wsm[(mf * 8 + g) * G::LDW + h * G::HC + kk + t];
+            for (int mf = 0; mf < G::MF; ++mf)
+                a[mf] = (SM::NSLOT == 8) ? sm.red[pad_off(mf * 8 + g, h * G::HC + kk + t)]
+                                         : sm.Wsm[(mf * 8 + g) * G::LDW + h * G::HC + kk + t];
 #pragma unroll
             for (int nf = 0; nf < G::NF; ++nf) {
                 if (KM && (rbase + nf * 8 + 8 <= kmin || rbase + nf * 8 >= kmax)) continue;
