@@ -349,7 +349,7 @@ def test_lookahead_off_bitwise_identical():
 def test_w16_update_matches_oracle_and_8warp_form(monkeypatch, m, n, nb, ib):
     """Bulk update with the 32-column slice over 16 warps (update_kernel16, default for nb >= 256)
     and over 8 warps (TQR_W16=0): both against the oracle (R, residual, thin-Q orthogonality,
-    least squares -- Q^T B runs the same kernels) and within rounding of each other.  n <= 1030:
+    least squares -- Q^T B runs the same kernels) and bitwise equal to each other.  n <= 1030:
     the absolute 1e-13 orthogonality bar is the one LAPACK meets there (reading Q19; at 2048^2 the
     16-warp form measured 1.13e-13 against LAPACK's 7.0e-14 on the same matrix, the 1.5-1.8x ratio
     of the full-size table, profiles/r02_full_parity.json)."""
@@ -371,7 +371,9 @@ def test_w16_update_matches_oracle_and_8warp_form(monkeypatch, m, n, nb, ib):
         np.testing.assert_allclose(to_np(Bd)[:n], oracle.solve_ls(A, B), rtol=1e-8, atol=1e-10)
         out[w16] = np.triu(Rg[:n])
         plan.close()
-    assert colnorm_rel_err(out["1"], out["0"]) <= 1e-12
+    # same rows per partial slot, same slot order, same DMMA order per accumulator: bitwise equal
+    # (which is what keeps the full-size parity of profiles/r02_full_parity.json valid for it)
+    assert np.array_equal(out["1"], out["0"])
 
 
 def test_repeat_factor_deterministic():
