@@ -432,15 +432,21 @@ __global__ void __launch_bounds__(kThreads, 1) update_kernel(UpdateArgs a) {
 }
 
 // ============================================================================ 16-warp bulk update
-// update_kernel's plain Q^T chain (nsteps = 1, no jobs, no flags) with the 32-column slice split over
-// 16 warps (tile_w16.cuh).
+// update_kernel's Q^T chain with the 32-column slice split over 16 warps (tile_w16.cuh): plain
+// launches and the forward wavefront of tqr_apply_qt (nsteps > 1: CTA = (step offset, slice), tile i
+// of step k only after the step-(k-1) CTA of the same slice has finished it; progress flags, lower
+// CTA index, so in-order dispatch cannot deadlock).  No jobs, no lookahead flags.
 template <int NB, int IB>
 __global__ void __launch_bounds__(kThreads16, 1) update_kernel16(UpdateArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     auto& sm = *reinterpret_cast<Smem16<NB, IB>*>(smem_raw);
     constexpr int SPG = NB / 32, NBLK = NB / IB;
-    const int k = a.k;
-    const int bid = (int)blockIdx.x;
+    const int st = a.nsteps > 1 ? (int)(blockIdx.x / a.nslc) : 0;
+    const int bid = a.nsteps > 1 ? (int)(blockIdx.x % a.nslc) : (int)blockIdx.x;
+    const int k = a.k + st;
+    const double* __restrict__ Vb = a.V + (int64_t)st * a.vcol;
+    const double* __restrict__ Tb = a.T + (int64_t)st * a.tcol;
+    const double* __restrict__ Eb = a.Vexp + (int64_t)st * a.ecol;
     const int grp = bid / SPG, c0 = (bid % SPG) * 32;
     double* Xg = a.X + (int64_t)(a.group0 + grp * a.gstride) * a.col_stride + (int64_t)c0 * a.ld;
     double* Xk = Xg + (int64_t)k * a.tile_stride;
@@ -455,15 +461,20 @@ __global__ void __launch_bounds__(kThreads16, 1) update_kernel16(UpdateArgs a) {
     const int ntiles = a.p - k - 1 + (a.do_unmqr ? 1 : 0);
     auto tile_of = [&](int q) -> int { return a.do_unmqr ? (q == 0 ? -1 : k + q) : k + 1 + q; };
     auto vblock = [&](int ti, int s) -> const double* {
-        return (ti < 0 ? a.Vexp : a.V + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;
+        return (ti < 0 ? Eb : Vb + (int64_t)ti * a.vstride * vtile) + (int64_t)s * IB * NB;
     };
     Slice16<NB, IB> X;
     if (ntiles > 0) stage16(sm, vblock(tile_of(0), 0), 0);
     for (int q = 0; q < ntiles; ++q) {
         const int ti = tile_of(q);
         double* Xi = (ti < 0) ? Xk : Xg + (int64_t)ti * a.tile_stride;
-        const double* Tt = a.T + (int64_t)(ti < 0 ? k : ti * a.vstride) * IB * NB;
-        X.load(Xi, a.ld);
+        const double* Tt = Tb + (int64_t)(ti < 0 ? k : ti * a.vstride) * IB * NB;
+        if (a.nsteps > 1) {
+            if (st > 0) flag_wait_geq(a.prog + (int64_t)(st - 1) * a.nslc + bid, (unsigned)((ti < 0 ? k : ti) - k + 2));
+            X.load_cg(Xi, a.ld);   // written by another CTA: L2, not a stale L1 line
+        } else {
+            X.load(Xi, a.ld);
+        }
         for (int s = 0; s < NBLK; ++s) {
             const double* nxt = nullptr;
             if (s + 1 < NBLK) nxt = vblock(ti, s + 1);
@@ -476,7 +487,9 @@ __global__ void __launch_bounds__(kThreads16, 1) update_kernel16(UpdateArgs a) {
                                              nxt, vph);
         }
         X.store(Xi, a.ld);
+        if (a.nsteps > 1) __threadfence();
         __syncthreads();   // row tile k (the X1 rows) is re-read by other threads
+        if (a.nsteps > 1 && threadIdx.x == 0) flag_release(a.prog + (int64_t)st * a.nslc + bid, (unsigned)(q + 1));
     }
 }
 
@@ -576,7 +589,7 @@ static cudaError_t launch_update_t(const UpdateArgs& a, int nslices, bool trans,
     if (grid <= 0) return cudaSuccess;
     if constexpr (W == 32 && NB >= 256) {
         // 16 warps per CTA for the plain Q^T chain (C5 1629 -> 1605 ms, C3 229 -> 226 ms)
-        if (a.w16 && trans && a.nsteps == 1 && a.domL == 0 && !a.wflags && !a.cflags) {
+        if (a.w16 && trans && a.domL == 0 && !a.wflags && !a.cflags) {
             const size_t sm16 = sizeof(Smem16<NB, IB>);
             auto kern = update_kernel16<NB, IB>;
             cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm16);

@@ -49,6 +49,16 @@ struct Slice16 {
                 acc[mf][nf][1] = v.y;
             }
     }
+    __device__ __forceinline__ void load_cg(const double* P, int64_t ld) {
+#pragma unroll
+        for (int mf = 0; mf < 2; ++mf)
+#pragma unroll
+            for (int nf = 0; nf < NF; ++nf) {
+                const double2 v = ld2_cg(P + (int64_t)(c0() + mf * 8) * ld + r0() + nf * 8);
+                acc[mf][nf][0] = v.x;
+                acc[mf][nf][1] = v.y;
+            }
+    }
     __device__ __forceinline__ void store(double* P, int64_t ld) const {
 #pragma unroll
         for (int mf = 0; mf < 2; ++mf)

@@ -2223,6 +2223,7 @@ static tqr_status apply_device(tqr_plan h, char trans, void* Bw, int64_t ldw, in
         u.group0 = 0; u.gstride = 1; u.k = k0; u.p = h->p; u.do_unmqr = 1;
         u.nsteps = q; u.nslc = (int)nslices; u.prog = (unsigned*)h->prog;
         u.vcol = p * h->vt; u.tcol = p * (int64_t)h->ib * nb; u.ecol = h->vt;
+        u.w16 = h->w16 ? 1 : 0;
         CUDA_TRY(h, tqr::launch_update(nb, h->ib, 32, u, (int)(q * nslices), fwd, s));
         h->launches++;
         return TQR_OK;
