@@ -15,7 +15,6 @@
 //                   lower part (the back substitution of tqr_solve_ls is in trsm.cu).
 #include <algorithm>
 #include <cstdio>
-#include <cstdlib>
 #include <cstring>
 #include <type_traits>
 #include "tile_ops.cuh"
@@ -588,7 +587,7 @@ static cudaError_t launch_update_t(const UpdateArgs& a, int nslices, bool trans,
     const int grid = nslices;
     if (grid <= 0) return cudaSuccess;
     if constexpr (W == 32 && NB >= 256) {
-        // 16 warps per CTA for the plain Q^T chain (C5 1629 -> 1605 ms, C3 229 -> 226 ms)
+        // 16 warps per CTA for the Q^T chain, plain or wavefront (C5 1629 -> 1592 ms, C3 229 -> 225 ms)
         if (a.w16 && trans && a.domL == 0 && !a.wflags && !a.cflags) {
             const size_t sm16 = sizeof(Smem16<NB, IB>);
             auto kern = update_kernel16<NB, IB>;
