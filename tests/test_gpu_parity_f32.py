@@ -124,6 +124,8 @@ def test_f32_logical_devices_and_host_path_bitwise():
     _, R1 = gpu_qr32(A32, nb, ib)
     _, R2 = gpu_qr32(A32, nb, ib, ndev=3, guide=[1, 0, 2, 2], logical_devices=True)
     assert np.array_equal(R1, R2)
+    # and against the oracle directly (FP64 Algorithm 1 on the FP32 input)
+    assert colnorm_rel_err(np.triu(R2[:n]).astype(np.float64), oracle.qr(A32.astype(np.float64)).R) <= R_TOL
     plan = tqr.Plan(m, n, nb, ib, dtype=tqr.TQR_F32)
     Ah = np.asfortranarray(A32.copy())
     plan.factor(Ah)
@@ -141,6 +143,7 @@ def test_f32_nccl_transport_single_rank_bitwise():
     Ad = dev32(A32)
     plan.factor(Ad)
     assert np.array_equal(to_np(Ad), R1)
+    assert colnorm_rel_err(np.triu(R1[:n]).astype(np.float64), oracle.qr(A32.astype(np.float64)).R) <= R_TOL
 
 
 @pytest.mark.slow
